@@ -1,0 +1,196 @@
+/*
+ * abs.h — C ABI of the B200-native Adaptive Bulk Search (ABS) hot path.
+ *
+ * Method: Yasudo, Nakano, Ito, Tatekawa, Katsuki, Yazane, Inaba, "Adaptive
+ * Bulk Search: Solving Quadratic Unconstrained Binary Optimization Problems
+ * on Multiple GPUs", ICPP 2020.  Citations "P:Lnnn" are line numbers of
+ * /root/reference/PAPER.md; "reading Cnn" refers to DESIGN.md §Readings.
+ *
+ * Problem: given an n x n symmetric int16 weight matrix W, find an
+ * n-bit vector X minimising E(X) = X^T W X = sum_{i,j} W_ij x_i x_j (Eq.(1)).
+ *
+ * Conventions shared by every call:
+ *   - Bit vectors: bit i of X is bit (i & 31) of uint32 word (i >> 5); a vector
+ *     has words(n) = ceil(n / 32) words; on input bits >= n are ignored, on
+ *     output they are 0.
+ *   - Energies are int64 (P:L519 prints -33,115,098,990 > 2^31); per-bit
+ *     deltas Delta_i(X) = E(flip_i X) - E(X) (Eq.(11)) are int32,
+ *     exact for n <= 32768 (reading C12).
+ *   - Every call returns ABS_OK (0) or a negative ABS_E* code; no C++
+ *     exception crosses the ABI.  A context is NOT thread-safe: one caller
+ *     thread per context.  The library owns its CUDA streams, device memory
+ *     and (async mode) its host GA thread.
+ *   - "Host" pointers are ordinary CPU memory owned by the caller; the
+ *     library copies what it needs before returning.  Calls whose names end
+ *     in _dev take CUDA device pointers on the context's device.
+ *   - There is no CPU fallback: a context can only be created on a CUDA
+ *     device of compute capability 10.0 (B200, sm_100a); otherwise
+ *     abs_create returns ABS_ECUDA.
+ */
+#ifndef ABS_H
+#define ABS_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#if defined(__GNUC__)
+#define ABS_API __attribute__((visibility("default")))
+#else
+#define ABS_API
+#endif
+
+#define ABS_OK 0
+#define ABS_EINVAL (-1)   /* bad argument (n out of range, W not symmetric, NULL, ...) */
+#define ABS_ENOMEM (-2)   /* host or device allocation failed */
+#define ABS_ECUDA (-3)    /* CUDA runtime error or no sm_100 device */
+#define ABS_ESTATE (-5)   /* call not valid in the current state */
+#define ABS_EEMPTY (-6)   /* no finite-energy solution in the pool yet */
+#define ABS_ERANGE (-7)   /* a Delta left the int32 range (cannot happen for n <= 32768) */
+
+#define ABS_N_MAX 32768   /* 32k bits, P:L23 / P:L416 */
+#define ABS_LADDER_MAX 32
+
+/* Search modes. */
+#define ABS_MODE_LOCKSTEP 0 /* deterministic: every search runs one round per
+                             * step, the host inserts all results in global
+                             * search-id order, then generates the next
+                             * targets.  Bit-exact with
+                             * the oracle. */
+#define ABS_MODE_ASYNC 1    /* the paper's system (Fig. 5): a
+                             * persistent kernel and a host GA thread exchange
+                             * targets and results through pinned buffers
+                             * without synchronising. */
+
+typedef struct abs_config {
+    int32_t searches;       /* searches run by this context (per GPU); 0 -> 148 */
+    int32_t search_offset;  /* global id of this context's first search
+                             * (multi-GPU partitioning) */
+    int64_t local_flips;    /* L: forced flips of the local search per round
+                             * ("fixed number of flips"); 0 -> n (reading C8) */
+    int32_t pool_size;      /* m: solutions kept by the host GA; 0 -> 64 */
+    int32_t ladder_len;     /* window lengths l ("temperature"):      */
+    int32_t ladder[ABS_LADDER_MAX]; /* search s uses ladder[s mod ladder_len];
+                             * ladder_len 0 -> {4,8,..,min(256,n/4)} (reading C7) */
+    uint64_t seed;          /* Philox key for the pool and GA draws */
+    int32_t p_cross;        /* per-mille; <0 -> 450 (reading C10) */
+    int32_t p_mut;          /* per-mille; <0 -> 450; copy = 1000 - p_cross - p_mut */
+    int32_t mut_max;        /* mutation flips 1 + (u mod mut_max) bits; 0 -> max(1, n/32) */
+    int32_t mode;           /* ABS_MODE_LOCKSTEP or ABS_MODE_ASYNC */
+    int32_t external_merge; /* lockstep only: 1 = do NOT insert this context's
+                             * results into its pool; the caller inserts the
+                             * results of all ranks with abs_pool_insert (in
+                             * global search-id order) before the next step */
+    int32_t device;         /* CUDA device ordinal; -1 -> current device */
+    int32_t reserved[8];    /* must be 0 */
+} abs_config;
+
+typedef struct abs_stats {
+    int64_t flips;            /* flips done by all searches (straight + local) */
+    int64_t straight_flips;   /* of which straight-search flips (Alg. 5) */
+    int64_t evaluated;        /* searched solutions = flips * n */
+    int64_t rounds;           /* completed rounds (device Steps 2-5), all searches */
+    double search_seconds;    /* device time inside abs_search (CUDA events) */
+    int64_t pool_inserted;    /* accepted pool insertions */
+    int32_t n;
+    int32_t n_pad;            /* padded length used on device (multiple of 1024) */
+    int32_t searches;
+    int32_t threads_per_search;
+    int64_t steps;            /* abs_search steps completed */
+    int64_t h2d_bytes;        /* bytes copied host->device by the library */
+    int64_t d2h_bytes;        /* bytes copied device->host by the library */
+    int64_t kernel_launches;  /* kernels launched by the library */
+    double step_seconds;      /* device time (CUDA events on the library stream)
+                               * from entry to exit of every abs_search call,
+                               * host GA gaps included */
+    int64_t round_kernel_launches; /* launches of the search (round) kernel */
+} abs_stats;
+
+typedef struct abs_ctx abs_ctx;
+
+/* Fill *cfg with defaults (all fields 0 / -1 as documented above). */
+ABS_API void abs_config_init(abs_config *cfg);
+
+/* Create a context for an instance.  W: host, row-major n x n
+ * int16, must be symmetric (W_ij = W_ji) else ABS_EINVAL; copied,
+ * caller keeps ownership.  1 <= n <= 32768.  cfg may be NULL (defaults).
+ * Every search starts from the zero vector with E = 0 and Delta_i = W_ii
+ * (device Step 1).  The pool starts as m Philox random bit
+ * vectors with E = +infinity (host Step 1). */
+ABS_API int abs_create(abs_ctx **out, int32_t n, const int16_t *W, const abs_config *cfg);
+
+/* As abs_create, but W is a device pointer (row-major n x n int16) on the
+ * configured device; it is copied, the caller keeps ownership. */
+ABS_API int abs_create_dev(abs_ctx **out, int32_t n, const int16_t *W_dev, const abs_config *cfg);
+
+/* Seed the host pool.  X == NULL: re-draw the Philox random pool with E =
+ * +infinity.  Otherwise X is `count` host bit vectors; their
+ * energies are computed ON THE DEVICE by the batched initialisation kernel
+ * (the host never computes an energy) and they are inserted with the
+ * pool rule (abs_pool_insert).  Valid before or between abs_search calls. */
+ABS_API int abs_seed_pool(abs_ctx *c, const uint32_t *X, int32_t count);
+
+/* Run `steps` steps (steps >= 0); blocks until done.
+ *   lockstep: each step = host GA generates one target per search from the
+ *     pool, every search runs one round — read target, reset best,
+ *     straight search C -> T, L window-policy local flips, emit (B, E_B)
+ *     (device Steps 2-5) — then the results are inserted in
+ *     search-id order (unless external_merge).
+ *   async: the persistent kernel runs until every search has emitted `steps`
+ *     more rounds; the host GA thread inserts results and writes new targets
+ *     while it runs. */
+ABS_API int abs_search(abs_ctx *c, int64_t steps);
+
+/* Best pool entry (pool[0]): X_out host (words(n) words), *E_out host.
+ * ABS_EEMPTY if no finite energy exists yet. */
+ABS_API int abs_best(const abs_ctx *c, uint32_t *X_out, int64_t *E_out);
+
+ABS_API int abs_stats_get(const abs_ctx *c, abs_stats *s);
+
+/* Top-k finite pool entries (ascending energy).  X_out: k*words(n) words,
+ * E_out: k.  *count_out = number written (<= k). */
+ABS_API int abs_pool_get(const abs_ctx *c, int32_t k, uint32_t *X_out, int64_t *E_out, int32_t *count_out);
+
+/* Insert `count` (X, E) pairs in the given order with the pool rule
+ * (P:L359): binary search on E; rejected if an entry with the same
+ * energy exists (reading C10) or E is not better than the worst entry;
+ * otherwise inserted in order and the worst entry dropped.  E must be the
+ * true energy of X (it is not recomputed).  *inserted_out may be NULL. */
+ABS_API int abs_pool_insert(abs_ctx *c, const uint32_t *X, const int64_t *E, int32_t count, int32_t *inserted_out);
+
+/* Batched initialisation: for `count` host bit vectors compute
+ * E (Eq.(1)) and, if delta_out != NULL, all Delta_i (Eq.(13)) on the
+ * device.  E_out: count int64; delta_out: count*n int32 (row-major). */
+ABS_API int abs_energy(abs_ctx *c, const uint32_t *X, int32_t count, int64_t *E_out, int32_t *delta_out);
+
+/* Lockstep: the (B, E_B) every local search emitted in the last step, in
+ * local search order.  B_out: searches*words(n) words, EB_out: searches. */
+ABS_API int abs_round_results(const abs_ctx *c, uint32_t *B_out, int64_t *EB_out);
+
+/* Lockstep: the targets T the searches used in the last step. */
+ABS_API int abs_round_targets(const abs_ctx *c, uint32_t *T_out);
+
+/* Per-search state (debug / parity): current solution C (words(n)), Delta
+ * (n int32), E, window offset a, window length l, FNV-1a-64 hash of the flip
+ * sequence (h = (h ^ k) * 0x100000001b3 from 0xcbf29ce484222325), flips.
+ * Any output pointer may be NULL.  `s` is the local search index. */
+ABS_API int abs_search_state(const abs_ctx *c, int32_t s, uint32_t *X_out, int32_t *delta_out, int64_t *E_out,
+                     int32_t *a_out, int32_t *l_out, uint64_t *hash_out, int64_t *flips_out);
+
+ABS_API void abs_destroy(abs_ctx *c);
+
+ABS_API const char *abs_strerror(int rc);
+
+/* Human-readable detail of the last error returned on the calling thread
+ * (never NULL; "" if none). */
+ABS_API const char *abs_last_error(void);
+
+/* Library version string. */
+ABS_API const char *abs_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ABS_H */

@@ -1,0 +1,293 @@
+"""Thin ctypes binding of libabs.so (include/abs.h).  Argument marshalling
+only: every step of the search runs in the library's sm_100a kernels and its
+host GA; there is no Python or CPU fallback.  Names follow the C ABI."""
+from __future__ import annotations
+
+import ctypes as C
+import os
+
+import numpy as np
+
+from . import build as _build
+
+ABS_OK = 0
+ABS_EINVAL = -1
+ABS_ENOMEM = -2
+ABS_ECUDA = -3
+ABS_ESTATE = -5
+ABS_EEMPTY = -6
+ABS_ERANGE = -7
+ABS_N_MAX = 32768
+ABS_LADDER_MAX = 32
+MODE_LOCKSTEP = 0
+MODE_ASYNC = 1
+
+
+class AbsError(RuntimeError):
+    def __init__(self, rc: int, where: str, detail: str):
+        super().__init__("%s failed: %s (%d): %s" % (where, _strerror(rc), rc, detail))
+        self.rc = rc
+
+
+class abs_config(C.Structure):
+    _fields_ = [
+        ("searches", C.c_int32),
+        ("search_offset", C.c_int32),
+        ("local_flips", C.c_int64),
+        ("pool_size", C.c_int32),
+        ("ladder_len", C.c_int32),
+        ("ladder", C.c_int32 * ABS_LADDER_MAX),
+        ("seed", C.c_uint64),
+        ("p_cross", C.c_int32),
+        ("p_mut", C.c_int32),
+        ("mut_max", C.c_int32),
+        ("mode", C.c_int32),
+        ("external_merge", C.c_int32),
+        ("device", C.c_int32),
+        ("reserved", C.c_int32 * 8),
+    ]
+
+
+class abs_stats(C.Structure):
+    _fields_ = [
+        ("flips", C.c_int64),
+        ("straight_flips", C.c_int64),
+        ("evaluated", C.c_int64),
+        ("rounds", C.c_int64),
+        ("search_seconds", C.c_double),
+        ("pool_inserted", C.c_int64),
+        ("n", C.c_int32),
+        ("n_pad", C.c_int32),
+        ("searches", C.c_int32),
+        ("threads_per_search", C.c_int32),
+        ("steps", C.c_int64),
+        ("h2d_bytes", C.c_int64),
+        ("d2h_bytes", C.c_int64),
+        ("kernel_launches", C.c_int64),
+        ("step_seconds", C.c_double),
+        ("round_kernel_launches", C.c_int64),
+    ]
+
+
+EXPORTS = [
+    "abs_config_init", "abs_create", "abs_create_dev", "abs_seed_pool", "abs_search", "abs_best",
+    "abs_stats_get", "abs_pool_get", "abs_pool_insert", "abs_energy", "abs_round_results",
+    "abs_round_targets", "abs_search_state", "abs_destroy", "abs_strerror", "abs_last_error", "abs_version",
+]
+
+_lib = None
+
+
+def library_path() -> str:
+    return _build.LIB
+
+
+def load(build_if_missing: bool = True):
+    """Load libabs.so (building it in-tree with nvcc if it is missing or stale)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    path = _build.LIB
+    if build_if_missing:
+        try:
+            path = _build.build()
+        except Exception as e:  # no nvcc: only an existing library can be used
+            if not os.path.exists(path):
+                raise ImportError("libabs.so is missing and cannot be built: %s" % e) from e
+    if not os.path.exists(path):
+        raise ImportError("libabs.so not found at %s (run paper_conf_icpp_yasudonitkyi20_b200/build.py)" % path)
+    L = C.CDLL(path)
+    P = C.POINTER
+    vp = C.c_void_p
+    L.abs_config_init.argtypes = [P(abs_config)]
+    L.abs_config_init.restype = None
+    L.abs_create.argtypes = [P(vp), C.c_int32, vp, P(abs_config)]
+    L.abs_create_dev.argtypes = [P(vp), C.c_int32, vp, P(abs_config)]
+    L.abs_seed_pool.argtypes = [vp, vp, C.c_int32]
+    L.abs_search.argtypes = [vp, C.c_int64]
+    L.abs_best.argtypes = [vp, vp, P(C.c_int64)]
+    L.abs_stats_get.argtypes = [vp, P(abs_stats)]
+    L.abs_pool_get.argtypes = [vp, C.c_int32, vp, vp, P(C.c_int32)]
+    L.abs_pool_insert.argtypes = [vp, vp, vp, C.c_int32, P(C.c_int32)]
+    L.abs_energy.argtypes = [vp, vp, C.c_int32, vp, vp]
+    L.abs_round_results.argtypes = [vp, vp, vp]
+    L.abs_round_targets.argtypes = [vp, vp]
+    L.abs_search_state.argtypes = [vp, C.c_int32, vp, vp, P(C.c_int64), P(C.c_int32), P(C.c_int32),
+                                   P(C.c_uint64), P(C.c_int64)]
+    L.abs_destroy.argtypes = [vp]
+    L.abs_destroy.restype = None
+    L.abs_strerror.argtypes = [C.c_int]
+    L.abs_strerror.restype = C.c_char_p
+    L.abs_last_error.argtypes = []
+    L.abs_last_error.restype = C.c_char_p
+    L.abs_version.argtypes = []
+    L.abs_version.restype = C.c_char_p
+    for name in EXPORTS:
+        fn = getattr(L, name)
+        if fn.restype is C.c_int:  # default restype
+            fn.restype = C.c_int
+    _lib = L
+    return L
+
+
+def _strerror(rc: int) -> str:
+    try:
+        return load(False).abs_strerror(rc).decode()
+    except Exception:
+        return "error"
+
+
+def _check(rc: int, where: str):
+    if rc != ABS_OK:
+        raise AbsError(rc, where, load().abs_last_error().decode())
+
+
+def _ptr(a):
+    return None if a is None else C.c_void_p(a.ctypes.data)
+
+
+def words(n: int) -> int:
+    return (int(n) + 31) // 32
+
+
+def make_config(n: int, searches: int = 148, search_offset: int = 0, local_flips: int | None = None,
+                pool_size: int = 64, ladder=None, seed: int = 1, p_cross: int = -1, p_mut: int = -1,
+                mut_max: int = 0, mode: int = MODE_LOCKSTEP, external_merge: bool = False,
+                device: int = -1) -> abs_config:
+    cfg = abs_config()
+    load().abs_config_init(C.byref(cfg))
+    cfg.searches = int(searches)
+    cfg.search_offset = int(search_offset)
+    cfg.local_flips = 0 if local_flips is None else int(local_flips)
+    cfg.pool_size = int(pool_size)
+    lad = list(ladder or [])
+    if len(lad) > ABS_LADDER_MAX:
+        raise ValueError("ladder too long")
+    cfg.ladder_len = len(lad)
+    for i, v in enumerate(lad):
+        cfg.ladder[i] = int(v)
+    cfg.seed = int(seed) & 0xFFFFFFFFFFFFFFFF
+    cfg.p_cross = int(p_cross)
+    cfg.p_mut = int(p_mut)
+    cfg.mut_max = int(mut_max)
+    cfg.mode = int(mode)
+    cfg.external_merge = 1 if external_merge else 0
+    cfg.device = int(device)
+    return cfg
+
+
+class Solver:
+    """One abs_ctx (one GPU / rank).  W: numpy int16 [n, n] (host) or a CUDA
+    torch.int16 tensor (device; abs_create_dev)."""
+
+    def __init__(self, W, **cfg_kwargs):
+        L = load()
+        self._c = C.c_void_p()
+        if hasattr(W, "is_cuda") and W.is_cuda:
+            import torch
+            assert W.dtype == torch.int16 and W.dim() == 2 and W.shape[0] == W.shape[1]
+            W = W.contiguous()
+            n = int(W.shape[0])
+            cfg_kwargs.setdefault("device", W.device.index if W.device.index is not None else torch.cuda.current_device())
+            self.cfg = make_config(n, **cfg_kwargs)
+            torch.cuda.synchronize(W.device)
+            _check(L.abs_create_dev(C.byref(self._c), n, C.c_void_p(W.data_ptr()), C.byref(self.cfg)), "abs_create_dev")
+        else:
+            W = np.ascontiguousarray(W, dtype=np.int16)
+            if W.ndim != 2 or W.shape[0] != W.shape[1]:
+                raise ValueError("W must be square")
+            n = int(W.shape[0])
+            self.cfg = make_config(n, **cfg_kwargs)
+            _check(L.abs_create(C.byref(self._c), n, _ptr(W), C.byref(self.cfg)), "abs_create")
+        self.n = n
+        self.words = words(n)
+        st = self.stats()
+        self.searches = st["searches"]
+
+    # -- lifecycle
+    def close(self):
+        if self._c:
+            load().abs_destroy(self._c)
+            self._c = C.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    # -- calls
+    def seed_pool(self, X=None):
+        if X is None:
+            _check(load().abs_seed_pool(self._c, None, 0), "abs_seed_pool")
+        else:
+            X = np.ascontiguousarray(np.atleast_2d(X), dtype=np.uint32)
+            assert X.shape[1] == self.words
+            _check(load().abs_seed_pool(self._c, _ptr(X), X.shape[0]), "abs_seed_pool")
+
+    def search(self, steps: int):
+        _check(load().abs_search(self._c, int(steps)), "abs_search")
+
+    def best(self):
+        X = np.zeros(self.words, np.uint32)
+        E = C.c_int64()
+        _check(load().abs_best(self._c, _ptr(X), C.byref(E)), "abs_best")
+        return X, int(E.value)
+
+    def stats(self) -> dict:
+        s = abs_stats()
+        _check(load().abs_stats_get(self._c, C.byref(s)), "abs_stats_get")
+        return {k: getattr(s, k) for k, _ in abs_stats._fields_}
+
+    def pool(self, k: int):
+        X = np.zeros((k, self.words), np.uint32)
+        E = np.zeros(k, np.int64)
+        cnt = C.c_int32()
+        _check(load().abs_pool_get(self._c, int(k), _ptr(X), _ptr(E), C.byref(cnt)), "abs_pool_get")
+        return X[:cnt.value], E[:cnt.value]
+
+    def pool_insert(self, X, E) -> int:
+        X = np.ascontiguousarray(np.atleast_2d(X), dtype=np.uint32)
+        E = np.ascontiguousarray(np.atleast_1d(E), dtype=np.int64)
+        assert X.shape[0] == E.shape[0] and X.shape[1] == self.words
+        ins = C.c_int32()
+        _check(load().abs_pool_insert(self._c, _ptr(X), _ptr(E), X.shape[0], C.byref(ins)), "abs_pool_insert")
+        return int(ins.value)
+
+    def energy(self, X, want_delta: bool = False):
+        X = np.ascontiguousarray(np.atleast_2d(X), dtype=np.uint32)
+        assert X.shape[1] == self.words
+        cnt = X.shape[0]
+        E = np.zeros(cnt, np.int64)
+        D = np.zeros((cnt, self.n), np.int32) if want_delta else None
+        _check(load().abs_energy(self._c, _ptr(X), cnt, _ptr(E), _ptr(D)), "abs_energy")
+        return (E, D) if want_delta else E
+
+    def round_results(self):
+        B = np.zeros((self.searches, self.words), np.uint32)
+        EB = np.zeros(self.searches, np.int64)
+        _check(load().abs_round_results(self._c, _ptr(B), _ptr(EB)), "abs_round_results")
+        return B, EB
+
+    def round_targets(self):
+        T = np.zeros((self.searches, self.words), np.uint32)
+        _check(load().abs_round_targets(self._c, _ptr(T)), "abs_round_targets")
+        return T
+
+    def search_state(self, s: int) -> dict:
+        X = np.zeros(self.words, np.uint32)
+        D = np.zeros(self.n, np.int32)
+        E, a, l, h, f = C.c_int64(), C.c_int32(), C.c_int32(), C.c_uint64(), C.c_int64()
+        _check(load().abs_search_state(self._c, int(s), _ptr(X), _ptr(D), C.byref(E), C.byref(a), C.byref(l),
+                                       C.byref(h), C.byref(f)), "abs_search_state")
+        return dict(X=X, D=D, E=int(E.value), a=int(a.value), l=int(l.value), hash=int(h.value), flips=int(f.value))
+
+
+def version() -> str:
+    return load().abs_version().decode()

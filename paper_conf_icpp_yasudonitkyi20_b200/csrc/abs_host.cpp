@@ -1,0 +1,670 @@
+// Host side of libabs: context, device layout, host GA (pool + targets) and
+// the search drivers behind the C ABI of include/abs.h.
+// Citations: /root/reference/PAPER.md line numbers (P:Lnnn); readings Cnn in DESIGN.md.
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <climits>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <thread>
+#include <vector>
+
+#include "abs.h"
+#include "abs_internal.h"
+#include "philox.hpp"
+
+namespace absb {
+
+constexpr uint32_t kTagPool = 0x504F4F4Cu;  // 'POOL'
+constexpr uint32_t kTagGA = 0x47415447u;    // 'GATG'
+constexpr int64_t kEInf = INT64_MAX;        // "+infinity" energy
+
+thread_local std::string g_last_error;
+
+static int fail(int rc, const std::string &what)
+{
+    g_last_error = what;
+    return rc;
+}
+
+#define ABS_CU(expr)                                                                                 \
+    do {                                                                                             \
+        cudaError_t e_ = (expr);                                                                     \
+        if (e_ != cudaSuccess)                                                                       \
+            return ::absb::fail(ABS_ECUDA, std::string(#expr) + ": " + cudaGetErrorString(e_));      \
+    } while (0)
+
+#define ABS_CK(expr)                                                                                 \
+    do {                                                                                             \
+        int e_ = (expr);                                                                             \
+        if (e_ != 0)                                                                                 \
+            return ::absb::fail(ABS_ECUDA, std::string(#expr) + ": " +                               \
+                                               cudaGetErrorString(static_cast<cudaError_t>(e_)));    \
+    } while (0)
+
+static int words_of(int n) { return (n + 31) / 32; }
+
+// ------------------------------------------------------------------ solution pool
+struct Pool {
+    int n = 0, m = 0, words = 0;
+    std::vector<int64_t> E;   // ascending; distinct finite values; +inf entries last
+    std::vector<uint32_t> X;  // m x words
+
+    void init(int n_, int m_) {
+        n = n_; m = m_; words = words_of(n_);
+        E.assign(m, kEInf);
+        X.assign((size_t)m * words, 0u);
+    }
+    // Host Step 1: random bit vectors with energy +infinity.
+    void randomize(uint64_t seed) {
+        const Philox4x32x10 rng(seed);
+        for (int e = 0; e < m; ++e) {
+            uint32_t *x = &X[(size_t)e * words];
+            for (int q = 0; 4 * q < words; ++q) {
+                const auto blk = rng({static_cast<uint32_t>(q), static_cast<uint32_t>(e), 0u, kTagPool});
+                for (int u = 0; u < 4 && 4 * q + u < words; ++u) x[4 * q + u] = blk[u];
+            }
+            if (n % 32) x[words - 1] &= (1u << (n % 32)) - 1u;
+            E[e] = kEInf;
+        }
+    }
+    // Distinct sorted insert, reading C10: same energy = same solution.
+    bool insert(const uint32_t *x, int64_t e) {
+        const auto it = std::lower_bound(E.begin(), E.end(), e);
+        const size_t pos = (size_t)(it - E.begin());
+        if (pos == (size_t)m) return false;
+        if (E[pos] == e && e != kEInf) return false;
+        // the worst solution is replaced
+        std::move_backward(E.begin() + pos, E.end() - 1, E.end());
+        std::move_backward(X.begin() + pos * words, X.end() - words, X.end());
+        E[pos] = e;
+        std::copy(x, x + words, X.begin() + pos * words);
+        return true;
+    }
+    int finite() const {
+        return (int)(std::lower_bound(E.begin(), E.end(), kEInf) - E.begin());
+    }
+};
+
+struct GaParams {
+    uint64_t seed = 1;
+    int p_cross = 450, p_mut = 450, mut_max = 1;
+};
+
+// New target for (round r, search sid): mutation / crossover / copy,
+// parents uniform over the pool (reading C10).  T must hold words(n) words.
+static void ga_target(const Pool &P, const GaParams &ga, int64_t r, int64_t sid, uint32_t *T)
+{
+    const Philox4x32x10 rng(ga.seed);
+    const uint32_t c1 = static_cast<uint32_t>(sid), c2 = static_cast<uint32_t>(r);
+    const auto head = rng({0u, c1, c2, kTagGA});
+    const uint32_t choice = head[0] % 1000u;
+    const uint32_t *p1 = &P.X[(size_t)(head[1] % (uint32_t)P.m) * P.words];
+    const uint32_t *p2 = &P.X[(size_t)(head[2] % (uint32_t)P.m) * P.words];
+    if (choice < (uint32_t)ga.p_cross) {
+        // crossover: each bit from either parent
+        Philox4x32x10::Block blk{};
+        for (int w = 0; w < P.words; ++w) {
+            if ((w & 3) == 0) blk = rng({1u + (uint32_t)(w >> 2), c1, c2, kTagGA});
+            const uint32_t take2 = blk[w & 3];
+            T[w] = (p1[w] & ~take2) | (p2[w] & take2);
+        }
+    } else if (choice < (uint32_t)(ga.p_cross + ga.p_mut)) {
+        // mutation: flip some random bits
+        std::copy(p1, p1 + P.words, T);
+        const uint32_t flips = 1u + head[3] % (uint32_t)std::max(1, ga.mut_max);
+        Philox4x32x10::Block blk{};
+        for (uint32_t f = 0; f < flips; ++f) {
+            if ((f & 3u) == 0) blk = rng({1u + (f >> 2), c1, c2, kTagGA});
+            const uint32_t bit = blk[f & 3u] % (uint32_t)P.n;
+            T[bit >> 5] ^= 1u << (bit & 31);
+        }
+    } else {
+        std::copy(p1, p1 + P.words, T);  // copy
+    }
+}
+
+}  // namespace absb
+
+using namespace absb;
+
+struct abs_ctx {
+    abs_config cfg{};
+    int device = 0;
+    cudaStream_t st = nullptr;
+    cudaEvent_t ev0 = nullptr, ev1 = nullptr, evs0 = nullptr, evs1 = nullptr;
+    Instance I;
+    SearchState S;
+    int64_t L = 0;
+    Pool pool;
+    GaParams ga;
+    int64_t round = 0;        // lockstep: rounds done (identical on every rank)
+    int bytes_per_vec = 0;    // n_pad / 8
+    // pinned host staging
+    uint8_t *T_h = nullptr, *B_h = nullptr;
+    int64_t *EB_h = nullptr;
+    bool have_results = false;
+    // stats
+    double search_seconds = 0.0;
+    int64_t rounds_done = 0, pool_inserted = 0, steps = 0;
+    int64_t h2d = 0, d2h = 0, launches = 0, round_launches = 0;
+    double step_seconds = 0.0;
+};
+
+static void free_ctx(abs_ctx *c)
+{
+    if (!c) return;
+    if (c->device >= 0) cudaSetDevice(c->device);
+    if (c->st) cudaStreamSynchronize(c->st);
+    cudaFree(c->I.Wz);
+    cudaFree(c->I.diag);
+    cudaFree(c->S.g);
+    cudaFree(c->S.X);
+    cudaFree(c->S.B);
+    cudaFree(c->S.T);
+    cudaFree(c->S.E);
+    cudaFree(c->S.EB);
+    cudaFree(c->S.a);
+    cudaFree(c->S.l);
+    cudaFree(c->S.hash);
+    cudaFree(c->S.flips);
+    cudaFree(c->S.sflips);
+    if (c->T_h) cudaFreeHost(c->T_h);
+    if (c->B_h) cudaFreeHost(c->B_h);
+    if (c->EB_h) cudaFreeHost(c->EB_h);
+    if (c->ev0) cudaEventDestroy(c->ev0);
+    if (c->ev1) cudaEventDestroy(c->ev1);
+    if (c->evs0) cudaEventDestroy(c->evs0);
+    if (c->evs1) cudaEventDestroy(c->evs1);
+    if (c->st) cudaStreamDestroy(c->st);
+    delete c;
+}
+
+static std::vector<int32_t> default_ladder(int n)
+{
+    // reading C7: {4, 8, ..., min(256, n/4)}
+    const int top = std::min(256, std::max(1, n / 4));
+    std::vector<int32_t> lad;
+    for (int v = 4; v <= top; v *= 2) lad.push_back(v);
+    if (lad.empty()) lad.push_back(std::max(1, top));
+    return lad;
+}
+
+// bit vectors: ABI words(n) uint32 <-> device bytes [n_pad/8] (little-endian, same bytes)
+static void words_to_bytes(const uint32_t *w, int words, uint8_t *dst, int bytes, int n)
+{
+    std::memset(dst, 0, (size_t)bytes);
+    std::memcpy(dst, w, sizeof(uint32_t) * (size_t)words);
+    if (n % 32) {
+        uint32_t last;
+        std::memcpy(&last, dst + 4 * (words - 1), 4);
+        last &= (1u << (n % 32)) - 1u;
+        std::memcpy(dst + 4 * (words - 1), &last, 4);
+    }
+}
+
+static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_device, const abs_config *cfg_in)
+{
+    if (!out) return fail(ABS_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (n < 1 || n > ABS_N_MAX) return fail(ABS_EINVAL, "n must be in [1, 32768]");
+    if (!W) return fail(ABS_EINVAL, "W is NULL");
+    abs_config cfg;
+    abs_config_init(&cfg);
+    if (cfg_in) cfg = *cfg_in;
+    if (cfg.searches == 0) cfg.searches = 148;
+    if (cfg.searches < 0 || cfg.search_offset < 0) return fail(ABS_EINVAL, "bad searches/search_offset");
+    if (cfg.local_flips == 0) cfg.local_flips = n;  // reading C8
+    if (cfg.local_flips < 0 || cfg.local_flips > INT32_MAX) return fail(ABS_EINVAL, "bad local_flips");
+    if (cfg.pool_size == 0) cfg.pool_size = 64;
+    if (cfg.pool_size < 1) return fail(ABS_EINVAL, "bad pool_size");
+    if (cfg.ladder_len < 0 || cfg.ladder_len > ABS_LADDER_MAX) return fail(ABS_EINVAL, "bad ladder_len");
+    if (cfg.p_cross < 0) cfg.p_cross = 450;
+    if (cfg.p_mut < 0) cfg.p_mut = 450;
+    if (cfg.p_cross + cfg.p_mut > 1000) return fail(ABS_EINVAL, "p_cross + p_mut > 1000");
+    if (cfg.mut_max == 0) cfg.mut_max = std::max(1, n / 32);
+    if (cfg.mut_max < 0) return fail(ABS_EINVAL, "bad mut_max");
+    if (cfg.mode != ABS_MODE_LOCKSTEP && cfg.mode != ABS_MODE_ASYNC) return fail(ABS_EINVAL, "bad mode");
+    std::vector<int32_t> ladder;
+    if (cfg.ladder_len == 0) {
+        ladder = default_ladder(n);
+    } else {
+        for (int i = 0; i < cfg.ladder_len; ++i) {
+            if (cfg.ladder[i] < 1) return fail(ABS_EINVAL, "ladder entries must be >= 1");
+            ladder.push_back(std::min(cfg.ladder[i], n));
+        }
+    }
+    cfg.ladder_len = (int)ladder.size();
+    for (int i = 0; i < cfg.ladder_len; ++i) cfg.ladder[i] = ladder[i];
+
+    int dev = cfg.device;
+    if (dev < 0) ABS_CU(cudaGetDevice(&dev));
+    ABS_CU(cudaSetDevice(dev));
+    cudaDeviceProp prop;
+    ABS_CU(cudaGetDeviceProperties(&prop, dev));
+    if (prop.major != 10) return fail(ABS_ECUDA, "libabs is built for sm_100a (B200); device is sm_" +
+                                                     std::to_string(prop.major) + std::to_string(prop.minor));
+
+    abs_ctx *c = new (std::nothrow) abs_ctx();
+    if (!c) return fail(ABS_ENOMEM, "host allocation");
+    c->cfg = cfg;
+    c->device = dev;
+    c->L = cfg.local_flips;
+    c->ga.seed = cfg.seed;
+    c->ga.p_cross = cfg.p_cross;
+    c->ga.p_mut = cfg.p_mut;
+    c->ga.mut_max = cfg.mut_max;
+
+    auto bail = [&](int rc) {
+        free_ctx(c);
+        return rc;
+    };
+#define CTX_CU(expr)                                                                                         \
+    do {                                                                                                     \
+        cudaError_t e_ = (expr);                                                                             \
+        if (e_ != cudaSuccess) return bail(fail(e_ == cudaErrorMemoryAllocation ? ABS_ENOMEM : ABS_ECUDA,    \
+                                                std::string(#expr) + ": " + cudaGetErrorString(e_)));        \
+    } while (0)
+
+    CTX_CU(cudaStreamCreateWithFlags(&c->st, cudaStreamNonBlocking));
+    CTX_CU(cudaEventCreate(&c->ev0));
+    CTX_CU(cudaEventCreate(&c->ev1));
+    CTX_CU(cudaEventCreate(&c->evs0));
+    CTX_CU(cudaEventCreate(&c->evs1));
+
+    // ---- instance layout
+    Instance &I = c->I;
+    I.n = n;
+    I.n_pad = ((n + 1023) / 1024) * 1024;
+    I.nt = I.n_pad / kBitsPerThread;
+    c->bytes_per_vec = I.n_pad / 8;
+    CTX_CU(cudaMalloc(&I.Wz, (size_t)I.n_pad * I.n_pad * sizeof(int16_t)));
+    CTX_CU(cudaMalloc(&I.diag, (size_t)I.n_pad * sizeof(int32_t)));
+    {
+        int16_t *W_in = nullptr;
+        const size_t wbytes = (size_t)n * n * sizeof(int16_t);
+        if (W_on_device) {
+            W_in = const_cast<int16_t *>(W);
+        } else {
+            CTX_CU(cudaMalloc(&W_in, wbytes));
+            CTX_CU(cudaMemcpyAsync(W_in, W, wbytes, cudaMemcpyHostToDevice, c->st));
+            c->h2d += (int64_t)wbytes;
+        }
+        unsigned long long *asym = nullptr;
+        CTX_CU(cudaMalloc(&asym, sizeof(unsigned long long)));
+        CTX_CU(cudaMemsetAsync(asym, 0, sizeof(unsigned long long), c->st));
+        const int rc = launch_prepare_w(W_in, n, I.n_pad, I.Wz, I.diag, asym, c->st);
+        c->launches++;
+        unsigned long long bad = 0;
+        cudaError_t e2 = cudaMemcpyAsync(&bad, asym, sizeof(bad), cudaMemcpyDeviceToHost, c->st);
+        cudaError_t e3 = cudaStreamSynchronize(c->st);
+        cudaFree(asym);
+        if (!W_on_device) cudaFree(W_in);
+        if (rc) return bail(fail(ABS_ECUDA, std::string("prepare_w: ") + cudaGetErrorString((cudaError_t)rc)));
+        CTX_CU(e2);
+        CTX_CU(e3);
+        if (bad) return bail(fail(ABS_EINVAL, "W is not symmetric (" + std::to_string(bad) + " entries)"));
+    }
+
+    // ---- per-search state
+    SearchState &S = c->S;
+    S.S = cfg.searches;
+    const size_t Sn = (size_t)std::max(1, S.S);
+    CTX_CU(cudaMalloc(&S.g, Sn * 32 * I.nt * sizeof(int32_t)));
+    CTX_CU(cudaMalloc(&S.X, Sn * c->bytes_per_vec));
+    CTX_CU(cudaMalloc(&S.B, Sn * c->bytes_per_vec));
+    CTX_CU(cudaMalloc(&S.T, Sn * c->bytes_per_vec));
+    CTX_CU(cudaMalloc(&S.E, Sn * sizeof(int64_t)));
+    CTX_CU(cudaMalloc(&S.EB, Sn * sizeof(int64_t)));
+    CTX_CU(cudaMalloc(&S.a, Sn * sizeof(int32_t)));
+    CTX_CU(cudaMalloc(&S.l, Sn * sizeof(int32_t)));
+    CTX_CU(cudaMalloc(&S.hash, Sn * sizeof(uint64_t)));
+    CTX_CU(cudaMalloc(&S.flips, Sn * sizeof(int64_t)));
+    CTX_CU(cudaMalloc(&S.sflips, Sn * sizeof(int64_t)));
+    {
+        std::vector<int32_t> lv(Sn);
+        for (size_t s = 0; s < Sn; ++s) lv[s] = ladder[(size_t)(cfg.search_offset + s) % ladder.size()];
+        CTX_CU(cudaMemcpyAsync(S.l, lv.data(), Sn * sizeof(int32_t), cudaMemcpyHostToDevice, c->st));
+        c->h2d += (int64_t)(Sn * sizeof(int32_t));
+    }
+    {
+        const int rc = launch_zero_start(I, S, 0, S.S, c->st);  // device Step 1
+        c->launches++;
+        if (rc) return bail(fail(ABS_ECUDA, std::string("zero_start: ") + cudaGetErrorString((cudaError_t)rc)));
+    }
+    CTX_CU(cudaMemsetAsync(S.T, 0, Sn * c->bytes_per_vec, c->st));
+    CTX_CU(cudaMallocHost(&c->T_h, Sn * c->bytes_per_vec));
+    CTX_CU(cudaMallocHost(&c->B_h, Sn * c->bytes_per_vec));
+    CTX_CU(cudaMallocHost(&c->EB_h, Sn * sizeof(int64_t)));
+    std::memset(c->T_h, 0, Sn * c->bytes_per_vec);
+    CTX_CU(cudaStreamSynchronize(c->st));
+
+    // ---- host GA pool (host Step 1)
+    c->pool.init(n, cfg.pool_size);
+    c->pool.randomize(cfg.seed);
+#undef CTX_CU
+    *out = c;
+    return ABS_OK;
+}
+
+// One lockstep step: targets, one round per search, inserts.
+static int lockstep_step(abs_ctx *c)
+{
+    const int S = c->S.S, words = c->pool.words, bpv = c->bytes_per_vec;
+    // host Step 4: "generates ... new target solutions by GA"
+    std::vector<uint32_t> T(words);
+    for (int s = 0; s < S; ++s) {
+        ga_target(c->pool, c->ga, c->round, (int64_t)c->cfg.search_offset + s, T.data());
+        std::memcpy(c->T_h + (size_t)s * bpv, T.data(), sizeof(uint32_t) * words);
+    }
+    ABS_CU(cudaMemcpyAsync(c->S.T, c->T_h, (size_t)S * bpv, cudaMemcpyHostToDevice, c->st));
+    c->h2d += (int64_t)S * bpv;
+    RoundArgs a{};
+    a.Wz = c->I.Wz;
+    a.n = c->I.n;
+    a.n_pad = c->I.n_pad;
+    a.nt = c->I.nt;
+    a.g = c->S.g;
+    a.X = c->S.X;
+    a.T = c->S.T;
+    a.B = c->S.B;
+    a.E = c->S.E;
+    a.EB = c->S.EB;
+    a.a = c->S.a;
+    a.l = c->S.l;
+    a.hash = c->S.hash;
+    a.flips = c->S.flips;
+    a.sflips = c->S.sflips;
+    a.L = c->L;
+    a.S = S;
+    ABS_CU(cudaEventRecord(c->ev0, c->st));
+    ABS_CK(launch_round(a, c->st));
+    c->launches++;
+    c->round_launches++;
+    ABS_CU(cudaEventRecord(c->ev1, c->st));
+    ABS_CU(cudaMemcpyAsync(c->B_h, c->S.B, (size_t)S * bpv, cudaMemcpyDeviceToHost, c->st));
+    ABS_CU(cudaMemcpyAsync(c->EB_h, c->S.EB, (size_t)S * sizeof(int64_t), cudaMemcpyDeviceToHost, c->st));
+    c->d2h += (int64_t)S * (bpv + 8);
+    ABS_CU(cudaStreamSynchronize(c->st));
+    float ms = 0.f;
+    ABS_CU(cudaEventElapsedTime(&ms, c->ev0, c->ev1));
+    c->search_seconds += ms * 1e-3;
+    c->have_results = true;
+    c->rounds_done += S;
+    if (!c->cfg.external_merge) {
+        // host Step 3: insert the new solutions (ascending search id)
+        for (int s = 0; s < S; ++s) {
+            std::memcpy(T.data(), c->B_h + (size_t)s * bpv, sizeof(uint32_t) * words);
+            c->pool_inserted += c->pool.insert(T.data(), c->EB_h[s]) ? 1 : 0;
+        }
+    }
+    c->round += 1;
+    c->steps += 1;
+    return ABS_OK;
+}
+
+extern "C" {
+
+void abs_config_init(abs_config *cfg)
+{
+    if (!cfg) return;
+    std::memset(cfg, 0, sizeof(*cfg));
+    cfg->seed = 1;
+    cfg->p_cross = -1;
+    cfg->p_mut = -1;
+    cfg->mode = ABS_MODE_LOCKSTEP;
+    cfg->device = -1;
+}
+
+int abs_create(abs_ctx **out, int32_t n, const int16_t *W, const abs_config *cfg)
+{
+    try {
+        return create_common(out, n, W, false, cfg);
+    } catch (const std::bad_alloc &) {
+        return fail(ABS_ENOMEM, "host allocation");
+    } catch (...) {
+        return fail(ABS_EINVAL, "unexpected exception");
+    }
+}
+
+int abs_create_dev(abs_ctx **out, int32_t n, const int16_t *W_dev, const abs_config *cfg)
+{
+    try {
+        return create_common(out, n, W_dev, true, cfg);
+    } catch (const std::bad_alloc &) {
+        return fail(ABS_ENOMEM, "host allocation");
+    } catch (...) {
+        return fail(ABS_EINVAL, "unexpected exception");
+    }
+}
+
+int abs_energy(abs_ctx *c, const uint32_t *X, int32_t count, int64_t *E_out, int32_t *delta_out)
+{
+    if (!c || (count > 0 && (!X || !E_out)) || count < 0) return fail(ABS_EINVAL, "bad arguments");
+    if (count == 0) return ABS_OK;
+    try {
+        ABS_CU(cudaSetDevice(c->device));
+        const int n = c->I.n, words = words_of(n), bpv = c->bytes_per_vec;
+        std::vector<uint8_t> xb((size_t)count * bpv);
+        for (int b = 0; b < count; ++b) words_to_bytes(X + (size_t)b * words, words, &xb[(size_t)b * bpv], bpv, n);
+        uint8_t *X_d = nullptr;
+        int64_t *E_d = nullptr;
+        int32_t *D_d = nullptr;
+        auto cleanup = [&]() {
+            cudaFree(X_d);
+            cudaFree(E_d);
+            cudaFree(D_d);
+        };
+        cudaError_t e = cudaMalloc(&X_d, xb.size());
+        if (e == cudaSuccess) e = cudaMalloc(&E_d, sizeof(int64_t) * (size_t)count);
+        if (e == cudaSuccess && delta_out) e = cudaMalloc(&D_d, sizeof(int32_t) * (size_t)count * n);
+        if (e == cudaSuccess) e = cudaMemcpyAsync(X_d, xb.data(), xb.size(), cudaMemcpyHostToDevice, c->st);
+        if (e == cudaSuccess) {
+            const int rc = launch_batch_init(c->I, X_d, count, E_d, D_d, c->st);
+            c->launches++;
+            e = (cudaError_t)rc;
+        }
+        if (e == cudaSuccess)
+            e = cudaMemcpyAsync(E_out, E_d, sizeof(int64_t) * (size_t)count, cudaMemcpyDeviceToHost, c->st);
+        if (e == cudaSuccess && delta_out)
+            e = cudaMemcpyAsync(delta_out, D_d, sizeof(int32_t) * (size_t)count * n, cudaMemcpyDeviceToHost, c->st);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(c->st);
+        cleanup();
+        c->h2d += (int64_t)xb.size();
+        c->d2h += (int64_t)count * 8 + (delta_out ? (int64_t)count * n * 4 : 0);
+        if (e != cudaSuccess) return fail(ABS_ECUDA, std::string("abs_energy: ") + cudaGetErrorString(e));
+        return ABS_OK;
+    } catch (const std::bad_alloc &) {
+        return fail(ABS_ENOMEM, "host allocation");
+    }
+}
+
+int abs_seed_pool(abs_ctx *c, const uint32_t *X, int32_t count)
+{
+    if (!c) return fail(ABS_EINVAL, "ctx is NULL");
+    if (!X) {
+        c->pool.randomize(c->cfg.seed);
+        return ABS_OK;
+    }
+    if (count < 0) return fail(ABS_EINVAL, "count < 0");
+    std::vector<int64_t> E((size_t)count);
+    // energies on the device: "a host never computes the energy function"
+    const int rc = abs_energy(c, X, count, E.data(), nullptr);
+    if (rc) return rc;
+    const int words = c->pool.words;
+    std::vector<uint32_t> x(words);
+    for (int b = 0; b < count; ++b) {
+        std::memcpy(x.data(), X + (size_t)b * words, sizeof(uint32_t) * words);
+        if (c->I.n % 32) x[words - 1] &= (1u << (c->I.n % 32)) - 1u;
+        c->pool_inserted += c->pool.insert(x.data(), E[b]) ? 1 : 0;
+    }
+    return ABS_OK;
+}
+
+int abs_search(abs_ctx *c, int64_t steps)
+{
+    if (!c || steps < 0) return fail(ABS_EINVAL, "bad arguments");
+    if (c->S.S == 0 || steps == 0) return ABS_OK;
+    try {
+        ABS_CU(cudaSetDevice(c->device));
+        if (c->cfg.mode != ABS_MODE_LOCKSTEP) return fail(ABS_EINVAL, "async mode not available in this build");
+        ABS_CU(cudaEventRecord(c->evs0, c->st));
+        for (int64_t s = 0; s < steps; ++s) {
+            const int rc = lockstep_step(c);
+            if (rc) return rc;
+        }
+        ABS_CU(cudaEventRecord(c->evs1, c->st));
+        ABS_CU(cudaEventSynchronize(c->evs1));
+        float ms = 0.f;
+        ABS_CU(cudaEventElapsedTime(&ms, c->evs0, c->evs1));
+        c->step_seconds += ms * 1e-3;
+        return ABS_OK;
+    } catch (const std::bad_alloc &) {
+        return fail(ABS_ENOMEM, "host allocation");
+    }
+}
+
+int abs_best(const abs_ctx *c, uint32_t *X_out, int64_t *E_out)
+{
+    if (!c || !X_out || !E_out) return fail(ABS_EINVAL, "bad arguments");
+    if (c->pool.finite() == 0) return fail(ABS_EEMPTY, "no finite energy in the pool");
+    std::memcpy(X_out, c->pool.X.data(), sizeof(uint32_t) * c->pool.words);
+    *E_out = c->pool.E[0];
+    return ABS_OK;
+}
+
+int abs_stats_get(const abs_ctx *c, abs_stats *s)
+{
+    if (!c || !s) return fail(ABS_EINVAL, "bad arguments");
+    std::memset(s, 0, sizeof(*s));
+    const int S = c->S.S;
+    if (S > 0) {
+        ABS_CU(cudaSetDevice(c->device));
+        std::vector<int64_t> f(S), sf(S);
+        ABS_CU(cudaMemcpy(f.data(), c->S.flips, sizeof(int64_t) * S, cudaMemcpyDeviceToHost));
+        ABS_CU(cudaMemcpy(sf.data(), c->S.sflips, sizeof(int64_t) * S, cudaMemcpyDeviceToHost));
+        for (int i = 0; i < S; ++i) {
+            s->flips += f[i];
+            s->straight_flips += sf[i];
+        }
+    }
+    s->evaluated = s->flips * (int64_t)c->I.n;
+    s->rounds = c->rounds_done;
+    s->search_seconds = c->search_seconds;
+    s->pool_inserted = c->pool_inserted;
+    s->n = c->I.n;
+    s->n_pad = c->I.n_pad;
+    s->searches = S;
+    s->threads_per_search = c->I.nt;
+    s->steps = c->steps;
+    s->h2d_bytes = c->h2d;
+    s->d2h_bytes = c->d2h;
+    s->kernel_launches = c->launches;
+    s->step_seconds = c->step_seconds;
+    s->round_kernel_launches = c->round_launches;
+    return ABS_OK;
+}
+
+int abs_pool_get(const abs_ctx *c, int32_t k, uint32_t *X_out, int64_t *E_out, int32_t *count_out)
+{
+    if (!c || k < 0 || (k > 0 && (!X_out || !E_out))) return fail(ABS_EINVAL, "bad arguments");
+    const int cnt = std::min(k, c->pool.finite());
+    std::memcpy(X_out, c->pool.X.data(), sizeof(uint32_t) * (size_t)cnt * c->pool.words);
+    std::memcpy(E_out, c->pool.E.data(), sizeof(int64_t) * (size_t)cnt);
+    if (count_out) *count_out = cnt;
+    return ABS_OK;
+}
+
+int abs_pool_insert(abs_ctx *c, const uint32_t *X, const int64_t *E, int32_t count, int32_t *inserted_out)
+{
+    if (!c || count < 0 || (count > 0 && (!X || !E))) return fail(ABS_EINVAL, "bad arguments");
+    const int words = c->pool.words;
+    std::vector<uint32_t> x(words);
+    int ins = 0;
+    for (int b = 0; b < count; ++b) {
+        std::memcpy(x.data(), X + (size_t)b * words, sizeof(uint32_t) * words);
+        if (c->I.n % 32) x[words - 1] &= (1u << (c->I.n % 32)) - 1u;
+        ins += c->pool.insert(x.data(), E[b]) ? 1 : 0;
+    }
+    c->pool_inserted += ins;
+    if (inserted_out) *inserted_out = ins;
+    return ABS_OK;
+}
+
+int abs_round_results(const abs_ctx *c, uint32_t *B_out, int64_t *EB_out)
+{
+    if (!c || !B_out || !EB_out) return fail(ABS_EINVAL, "bad arguments");
+    if (!c->have_results) return fail(ABS_ESTATE, "no round has run");
+    const int words = c->pool.words;
+    for (int s = 0; s < c->S.S; ++s) {
+        std::memcpy(B_out + (size_t)s * words, c->B_h + (size_t)s * c->bytes_per_vec, sizeof(uint32_t) * words);
+        EB_out[s] = c->EB_h[s];
+    }
+    return ABS_OK;
+}
+
+int abs_round_targets(const abs_ctx *c, uint32_t *T_out)
+{
+    if (!c || !T_out) return fail(ABS_EINVAL, "bad arguments");
+    if (!c->have_results) return fail(ABS_ESTATE, "no round has run");
+    const int words = c->pool.words;
+    for (int s = 0; s < c->S.S; ++s)
+        std::memcpy(T_out + (size_t)s * words, c->T_h + (size_t)s * c->bytes_per_vec, sizeof(uint32_t) * words);
+    return ABS_OK;
+}
+
+int abs_search_state(const abs_ctx *c, int32_t s, uint32_t *X_out, int32_t *delta_out, int64_t *E_out,
+                     int32_t *a_out, int32_t *l_out, uint64_t *hash_out, int64_t *flips_out)
+{
+    if (!c || s < 0 || s >= c->S.S) return fail(ABS_EINVAL, "bad arguments");
+    ABS_CU(cudaSetDevice(c->device));
+    const int n = c->I.n, nt = c->I.nt, bpv = c->bytes_per_vec, words = words_of(n);
+    std::vector<uint8_t> xb(bpv);
+    ABS_CU(cudaMemcpy(xb.data(), c->S.X + (size_t)s * bpv, bpv, cudaMemcpyDeviceToHost));
+    if (X_out) std::memcpy(X_out, xb.data(), sizeof(uint32_t) * words);
+    if (delta_out) {
+        std::vector<int32_t> g((size_t)32 * nt);
+        ABS_CU(cudaMemcpy(g.data(), c->S.g + (size_t)s * 32 * nt, sizeof(int32_t) * g.size(),
+                          cudaMemcpyDeviceToHost));
+        for (int i = 0; i < n; ++i) {
+            const int beta = i >> 3, t = beta % nt, slot = 8 * (beta / nt) + (i & 7);
+            const int gi = g[(size_t)slot * nt + t];
+            const int xi = (xb[i >> 3] >> (i & 7)) & 1;
+            delta_out[i] = xi ? -gi : gi;  // Delta_i = phi(x_i) g_i (Eq.(13))
+        }
+    }
+    int64_t v64;
+    int32_t v32;
+    uint64_t u64;
+    if (E_out) { ABS_CU(cudaMemcpy(&v64, c->S.E + s, 8, cudaMemcpyDeviceToHost)); *E_out = v64; }
+    if (a_out) { ABS_CU(cudaMemcpy(&v32, c->S.a + s, 4, cudaMemcpyDeviceToHost)); *a_out = v32; }
+    if (l_out) { ABS_CU(cudaMemcpy(&v32, c->S.l + s, 4, cudaMemcpyDeviceToHost)); *l_out = v32; }
+    if (hash_out) { ABS_CU(cudaMemcpy(&u64, c->S.hash + s, 8, cudaMemcpyDeviceToHost)); *hash_out = u64; }
+    if (flips_out) { ABS_CU(cudaMemcpy(&v64, c->S.flips + s, 8, cudaMemcpyDeviceToHost)); *flips_out = v64; }
+    return ABS_OK;
+}
+
+void abs_destroy(abs_ctx *c) { free_ctx(c); }
+
+const char *abs_strerror(int rc)
+{
+    switch (rc) {
+    case ABS_OK: return "ok";
+    case ABS_EINVAL: return "invalid argument";
+    case ABS_ENOMEM: return "out of memory";
+    case ABS_ECUDA: return "CUDA error";
+    case ABS_ESTATE: return "invalid state";
+    case ABS_EEMPTY: return "pool has no finite-energy solution";
+    case ABS_ERANGE: return "delta out of int32 range";
+    default: return "unknown error";
+    }
+}
+
+const char *abs_last_error(void) { return g_last_error.c_str(); }
+
+const char *abs_version(void) { return "abs-b200 0.1 (sm_100a)"; }
+
+}  // extern "C"

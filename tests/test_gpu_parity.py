@@ -1,0 +1,268 @@
+"""GPU parity: the CUDA path (libabs.so through its C ABI) against the CPU
+oracle on the same seeded inputs.  Integer method -> bit-exact everywhere:
+energies, Delta vectors, whole trajectories (FNV hash of the flip sequence,
+flip counts, window offsets), every emitted (B, E_B), the GA targets and the
+final pool."""
+from __future__ import annotations
+
+import itertools
+import time
+
+import numpy as np
+import pytest
+
+import oracle
+from workloads import maxcut_qubo, pack_bits, random_qubo, random_solutions, tsp_qubo
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():  # pragma: no cover
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+import paper_conf_icpp_yasudonitkyi20_b200 as abs_b200  # noqa: E402
+
+
+def make(W, **kw):
+    return abs_b200.Solver(W, **kw)
+
+
+def ocfg(n, searches, L, pool, seed, ladder=None, mut_max=None):
+    return oracle.Config(n=n, searches=searches, local_flips=L, pool_size=pool, seed=seed,
+                         ladder=list(ladder or []), mut_max=mut_max)
+
+
+def run_both(W, S, L, R, pool=16, seed=7, ladder=None, check_rounds=True):
+    n = W.shape[0]
+    s = make(W, searches=S, local_flips=L, pool_size=pool, seed=seed, ladder=ladder)
+    gB, gEB, gT = [], [], []
+    for _ in range(R):
+        s.search(1)
+        B, EB = s.round_results()
+        gB.append(B)
+        gEB.append(EB)
+        gT.append(s.round_targets())
+    o = oracle.run_lockstep(W, ocfg(n, S, L, pool, seed, ladder), R)
+    return s, o, np.array(gB), np.array(gEB), np.array(gT)
+
+
+def assert_same(s, o, gB, gEB, S, n, pool):
+    # every emitted result, every round
+    assert (gEB == o["EB"]).all(), "E_B differs"
+    assert (gB == o["B"]).all(), "B differs"
+    for i in range(S):
+        st = s.search_state(i)
+        assert st["flips"] == o["flips"][i], ("flips", i)
+        assert st["hash"] == int(o["hash"][i]), ("trajectory hash", i)
+        assert st["E"] == o["E"][i], ("E", i)
+        assert st["a"] == o["a"][i], ("offset", i)
+        assert (st["X"] == o["X"][i]).all(), ("X", i)
+        assert (st["D"].astype(np.int64) == o["D"][i]).all(), ("Delta", i)
+    PX, PE = s.pool(pool)
+    fin = o["poolE"] != oracle.EINF
+    assert (PE == o["poolE"][fin]).all()
+    assert (PX == o["poolX"][fin]).all()
+
+
+# ---------------------------------------------------------------- batched init
+@pytest.mark.parametrize("n", [1, 16, 33, 100, 1000, 1024, 1500, 2050])
+def test_batch_init_energy_and_delta(n):
+    W = random_qubo(n, n)
+    X = random_solutions(21, n, 5)            # spans two 16-solution tiles
+    X[0] = 0
+    X[1] = pack_bits(np.ones((1, n), bool))[0]  # all ones
+    s = make(W, searches=1)
+    Xdirty = X.copy()
+    Xdirty[1] = np.iinfo(np.uint32).max       # bits >= n must be ignored
+    E, D = s.energy(Xdirty, want_delta=True)
+    oD, oE = oracle.init_batch(W, X)
+    assert (E == oE).all()
+    assert (D.astype(np.int64) == oD).all()
+
+
+def test_batch_init_int32_extreme():
+    # reading C12: W == -32768, X = 1^n -> Delta_i = 32768 (2n - 1), the largest |Delta|
+    n = 4096
+    W = np.full((n, n), -32768, np.int16)
+    s = make(W, searches=1)
+    X = np.full((1, n // 32), 0xFFFFFFFF, np.uint32)
+    E, D = s.energy(X, want_delta=True)
+    assert (D == 32768 * (2 * n - 1)).all()
+    assert E[0] == -32768 * n * n
+
+
+def test_zero_start_state():
+    n = 1500
+    W = random_qubo(n, 3)
+    s = make(W, searches=3)
+    for i in range(3):
+        st = s.search_state(i)
+        assert st["E"] == 0 and st["flips"] == 0 and st["a"] == 0
+        assert (st["X"] == 0).all()
+        assert (st["D"] == np.diag(W)).all()
+
+
+def test_rejects_asymmetric_and_bad_n():
+    W = random_qubo(40, 1)
+    W[3, 5] += 1
+    with pytest.raises(abs_b200.AbsError) as e:
+        make(W, searches=1)
+    assert e.value.rc == abs_b200.ABS_EINVAL
+    with pytest.raises(abs_b200.AbsError):
+        make(np.zeros((0, 0), np.int16), searches=1)
+
+
+# ---------------------------------------------------------------- config 1 (n = 16)
+def test_config1_n16_bitexact_and_bruteforce():
+    n, S, L = 16, 256, 1000
+    W = random_qubo(n, 1)
+    s, o, gB, gEB, gT = run_both(W, S, L, 1, pool=32, seed=1)
+    assert_same(s, o, gB, gEB, S, n, 32)
+    allx = np.array(list(itertools.product([0, 1], repeat=n)), dtype=np.int64)
+    e_min = int(np.einsum("bi,ij,bj->b", allx, W.astype(np.int64), allx).min())
+    assert s.best()[1] == e_min
+
+
+# ---------------------------------------------------------------- lockstep trajectories
+@pytest.mark.parametrize("n,S,L,R,seed", [
+    (5, 8, 30, 3, 1),          # tiny, ragged word
+    (100, 12, 150, 3, 2),      # one warp, ragged
+    (1024, 6, 1024, 2, 3),     # config-2 size, one warp, full
+    (1100, 5, 300, 2, 4),      # 2 warps (n_pad 2048), ragged
+    (3000, 4, 500, 2, 5),      # 3 warps
+    (4100, 3, 400, 2, 6),      # NT = 160
+])
+def test_lockstep_random_qubo_bitexact(n, S, L, R, seed):
+    W = random_qubo(n, seed)
+    s, o, gB, gEB, gT = run_both(W, S, L, R, pool=8, seed=seed)
+    assert_same(s, o, gB, gEB, S, n, 8)
+
+
+def test_lockstep_maxcut_ties_bitexact():
+    # Max-Cut (Eq.(17)) with +-1 weights: deltas tie constantly -> exercises
+    # the lowest-index tie-break in every reduction (reading C5).
+    n = 2000
+    W = maxcut_qubo(n, 19990, seed=3)
+    s, o, gB, gEB, gT = run_both(W, 4, 600, 3, pool=8, seed=3)
+    assert_same(s, o, gB, gEB, 4, n, 8)
+
+
+def test_lockstep_tsp_bitexact():
+    c = 12
+    W = tsp_qubo(c, seed=2)
+    s, o, gB, gEB, gT = run_both(W, 6, 400, 3, pool=8, seed=2)
+    assert_same(s, o, gB, gEB, 6, c * c, 8)
+
+
+@pytest.mark.parametrize("ladder", [[1], [7], [64, 3], [100]])
+def test_lockstep_window_edge_cases(ladder):
+    # l = 1 (random-walk end), l not dividing n (wrap), l = n (greedy end)
+    n = 100
+    W = random_qubo(n, 11)
+    s, o, gB, gEB, gT = run_both(W, 4, 250, 2, pool=8, seed=11, ladder=ladder)
+    assert_same(s, o, gB, gEB, 4, n, 8)
+
+
+def test_lockstep_single_local_flip():
+    # L = 1: the round is almost only the straight search (Alg. 5)
+    n = 300
+    W = random_qubo(n, 12)
+    s, o, gB, gEB, gT = run_both(W, 5, 1, 3, pool=8, seed=12)
+    assert_same(s, o, gB, gEB, 5, n, 8)
+
+
+def test_targets_match_oracle_ga():
+    n = 200
+    W = random_qubo(n, 13)
+    s, o, gB, gEB, gT = run_both(W, 7, 50, 3, pool=6, seed=13)
+    p = oracle.Pool(n, 6, seed=13)
+    cfg = ocfg(n, 7, 50, 6, 13)
+    for r in range(3):
+        for i in range(7):
+            assert (gT[r, i] == p.target(cfg, r, i)).all()
+        for i in range(7):
+            p.insert(o["B"][r, i], o["EB"][r, i])
+
+
+def test_emitted_energies_are_true_energies():
+    n = 777
+    W = random_qubo(n, 14)
+    s = make(W, searches=9, local_flips=500, pool_size=8, seed=14)
+    s.search(2)
+    B, EB = s.round_results()
+    E = s.energy(B)
+    assert (E == EB).all()
+    for b in range(3):
+        assert oracle.energy(W, B[b]) == EB[b]
+
+
+def test_external_merge_equals_internal():
+    n = 500
+    W = random_qubo(n, 15)
+    a = make(W, searches=6, local_flips=200, pool_size=8, seed=15)
+    b = make(W, searches=6, local_flips=200, pool_size=8, seed=15, external_merge=True)
+    for _ in range(3):
+        a.search(1)
+        b.search(1)
+        B, EB = b.round_results()
+        b.pool_insert(B, EB)
+    assert (a.pool(8)[1] == b.pool(8)[1]).all()
+    assert (a.pool(8)[0] == b.pool(8)[0]).all()
+
+
+def test_sharded_ranks_equal_single_process():
+    """P14 / SURVEY §8(e): 3 'ranks' (contexts with search_offset) exchanging
+    all results each step reproduce the single-process oracle exactly."""
+    n, Sg, R, L = 300, 4, 3, 120
+    W = random_qubo(n, 16)
+    ranks = [make(W, searches=Sg, search_offset=r * Sg, local_flips=L, pool_size=8, seed=16, external_merge=True)
+             for r in range(3)]
+    for _ in range(R):
+        res = []
+        for s in ranks:
+            s.search(1)
+            res.append(s.round_results())
+        allB = np.concatenate([b for b, _ in res])
+        allE = np.concatenate([e for _, e in res])
+        for s in ranks:
+            s.pool_insert(allB, allE)
+    o = oracle.run_lockstep(W, ocfg(n, 3 * Sg, L, 8, 16), R)
+    for s in ranks:
+        PX, PE = s.pool(8)
+        assert (PE == o["poolE"]).all() and (PX == o["poolX"]).all()
+    for r, s in enumerate(ranks):
+        for i in range(Sg):
+            assert s.search_state(i)["hash"] == int(o["hash"][r * Sg + i])
+
+
+def test_seed_pool_uses_device_energies():
+    n = 250
+    W = random_qubo(n, 17)
+    s = make(W, searches=2, pool_size=4, seed=17)
+    X = random_solutions(6, n, 17)
+    s.seed_pool(X)
+    PX, PE = s.pool(4)
+    E_ref = np.array([oracle.energy(W, x) for x in X])
+    order = np.argsort(E_ref, kind="stable")[:4]
+    assert (PE == E_ref[order]).all()
+
+
+# ---------------------------------------------------------------- full size (bench launch configuration)
+def test_full_size_n32768_sampled():
+    """n = 32768 (config 5) in the launch configuration bench.py times
+    (one 1024-thread CTA per search), on 2 sampled searches with a reduced
+    L: trajectory hash, Delta, E, B, E_B identical to the oracle."""
+    n, S, L = 32768, 2, 64
+    W = random_qubo(n, 1)
+    t0 = time.time()
+    s = make(W, searches=S, local_flips=L, pool_size=4, seed=5)
+    s.search(1)
+    B, EB = s.round_results()
+    o = oracle.run_lockstep(W, ocfg(n, S, L, 4, 5), 1)
+    assert (EB == o["EB"][0]).all() and (B == o["B"][0]).all()
+    for i in range(S):
+        st = s.search_state(i)
+        assert st["hash"] == int(o["hash"][i]) and st["flips"] == o["flips"][i]
+        assert st["E"] == o["E"][i]
+        assert (st["D"].astype(np.int64) == o["D"][i]).all()
+    assert time.time() - t0 < 600
