@@ -12,8 +12,8 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libabs.so")
-SOURCES = ["abs_kernels.cu", "abs_host.cpp"]
-HEADERS = ["abs_internal.h", "philox.hpp"]
+SOURCES = ["abs_round.cu", "abs_setup.cu", "abs_host.cpp"]
+HEADERS = ["abs_internal.h", "philox.hpp", "ptx.cuh"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 

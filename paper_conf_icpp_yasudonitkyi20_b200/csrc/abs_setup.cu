@@ -1,0 +1,172 @@
+// sm_100a setup kernels of the ABS hot path: instance preparation, device
+// Step 1 (zero start) and the batched initialisation of Delta / E.
+// Citations: /root/reference/PAPER.md line numbers (P:Lnnn).
+#include <climits>
+#include <cstdint>
+
+#include "abs_internal.h"
+
+namespace absb {
+namespace {
+
+constexpr uint64_t kFnvOffset = 0xcbf29ce484222325ull;
+constexpr unsigned kFull = 0xffffffffu;
+
+// global bit index of slot s of thread t (see abs_internal.h)
+__device__ __forceinline__ int slot_index(int t, int nt, int s)
+{
+    return 8 * (t + nt * (s >> 3)) + (s & 7);
+}
+
+// ------------------------------------------------------------------ setup kernels
+// Wz = W with zero diagonal padded to n_pad x n_pad; diag = W_ii; counts
+// asymmetric entries (W must be symmetric).
+__global__ void prepare_w_kernel(const int16_t *__restrict__ W, int n, int n_pad, int16_t *__restrict__ Wz,
+                                 int32_t *__restrict__ diag, unsigned long long *asym)
+{
+    __shared__ int16_t ta[32][33];
+    __shared__ int16_t tb[32][33];
+    const int bx = blockIdx.x * 32, by = blockIdx.y * 32;
+    const int tx = threadIdx.x, ty = threadIdx.y;
+    for (int r = ty; r < 32; r += 8) {
+        const int row = by + r, col = bx + tx;
+        ta[r][tx] = (row < n && col < n) ? W[(size_t)row * n + col] : (int16_t)0;
+        const int row2 = bx + r, col2 = by + tx;  // transposed block
+        tb[r][tx] = (row2 < n && col2 < n) ? W[(size_t)row2 * n + col2] : (int16_t)0;
+    }
+    __syncthreads();
+    unsigned long long bad = 0;
+    for (int r = ty; r < 32; r += 8) {
+        const int row = by + r, col = bx + tx;
+        const int16_t v = ta[r][tx];
+        if (v != tb[tx][r]) ++bad;
+        Wz[(size_t)row * n_pad + col] = (row == col) ? (int16_t)0 : v;
+        if (row == col) diag[row] = (row < n) ? (int32_t)v : 0;
+    }
+    if (bad) atomicAdd(asym, bad);
+}
+
+// Device Step 1: C = 0, E = 0, Delta_i = W_ii (g_i = W_ii).
+__global__ void zero_start_kernel(int n, int nt, const int32_t *__restrict__ diag, int32_t *g, uint8_t *X,
+                                  uint8_t *B, int64_t *E, int64_t *EB, int32_t *a, uint64_t *hash, int64_t *flips,
+                                  int64_t *sflips, int s0)
+{
+    const int sid = s0 + blockIdx.x;
+    const int t = threadIdx.x;
+    int32_t *gs = g + (size_t)sid * 32 * nt;
+    for (int s = 0; s < 32; ++s) {
+        const int i = slot_index(t, nt, s);
+        gs[(size_t)s * nt + t] = (i < n) ? diag[i] : INT_MAX;  // pads are never candidates nor minima
+    }
+    for (int j = 0; j < 4; ++j) {
+        X[(size_t)sid * 4 * nt + t + nt * j] = 0;
+        B[(size_t)sid * 4 * nt + t + nt * j] = 0;
+    }
+    if (t == 0) {
+        E[sid] = 0;
+        EB[sid] = 0;
+        a[sid] = 0;  // reading C6
+        hash[sid] = kFnvOffset;
+        flips[sid] = 0;
+        sflips[sid] = 0;
+    }
+}
+
+// Batched initialisation.  Thread = column i, 16 solutions per
+// CTA row of the grid.  y_b = Wz x_b (Wz zero-diagonal), then
+//   g_i = 2 y_i + W_ii,  Delta_i = phi(x_i) g_i   (Eq.(13))
+//   E = sum_i x_i (y_i + W_ii)                    (Eq.(1))
+constexpr int kInitB = 16;
+constexpr int kInitT = 256;
+__global__ void __launch_bounds__(kInitT) batch_init_kernel(const int16_t *__restrict__ Wz,
+                                                            const int32_t *__restrict__ diag, int n, int n_pad,
+                                                            const uint8_t *__restrict__ X, int count,
+                                                            int64_t *__restrict__ Eout, int32_t *__restrict__ delta)
+{
+    extern __shared__ uint32_t sx[];  // [kInitB][n_pad/32]
+    __shared__ long long red[kInitB][kInitT / 32];
+    const int words = n_pad / 32;
+    const int b0 = blockIdx.y * kInitB;
+    const int i = blockIdx.x * kInitT + threadIdx.x;
+    for (int q = threadIdx.x; q < kInitB * words; q += kInitT) {
+        const int b = q / words, w = q % words;
+        uint32_t v = 0;
+        if (b0 + b < count) {
+            const uint8_t *xb = X + (size_t)(b0 + b) * (n_pad / 8) + 4 * w;
+            v = (uint32_t)xb[0] | ((uint32_t)xb[1] << 8) | ((uint32_t)xb[2] << 16) | ((uint32_t)xb[3] << 24);
+        }
+        sx[b * words + w] = v;
+    }
+    __syncthreads();
+    int acc[kInitB];
+#pragma unroll
+    for (int b = 0; b < kInitB; ++b) acc[b] = 0;
+    for (int w = 0; w < words; ++w) {
+        uint32_t xw[kInitB];
+        uint32_t any = 0;
+#pragma unroll
+        for (int b = 0; b < kInitB; ++b) {
+            xw[b] = sx[b * words + w];
+            any |= xw[b];
+        }
+        if (!any) continue;
+        for (int jj = 0; jj < 32; ++jj) {
+            const int j = w * 32 + jj;
+            const int v = Wz[(size_t)j * n_pad + i];  // column i of row j == W_ij (symmetric)
+#pragma unroll
+            for (int b = 0; b < kInitB; ++b)
+                if ((xw[b] >> jj) & 1u) acc[b] += v;
+        }
+    }
+    const int di = diag[i];
+    const uint32_t *xi_w = sx + (i >> 5);
+#pragma unroll
+    for (int b = 0; b < kInitB; ++b) {
+        const int xi = (int)((xi_w[b * words] >> (i & 31)) & 1u);
+        const int gi = 2 * acc[b] + di;
+        if (delta && i < n && b0 + b < count) delta[(size_t)(b0 + b) * n + i] = xi ? -gi : gi;
+        long long e = xi ? (long long)acc[b] + di : 0;
+        for (int o = 16; o > 0; o >>= 1) e += __shfl_xor_sync(kFull, e, o);
+        if ((threadIdx.x & 31) == 0) red[b][threadIdx.x >> 5] = e;
+    }
+    __syncthreads();
+    if (threadIdx.x < kInitB && b0 + (int)threadIdx.x < count) {
+        long long e = 0;
+        for (int w = 0; w < kInitT / 32; ++w) e += red[threadIdx.x][w];
+        atomicAdd(reinterpret_cast<unsigned long long *>(Eout + b0 + threadIdx.x), (unsigned long long)e);
+    }
+}
+
+}  // namespace
+
+
+// ------------------------------------------------------------------ launchers
+int launch_prepare_w(const int16_t *W_in, int32_t n, int32_t n_pad, int16_t *Wz, int32_t *diag,
+                     unsigned long long *asym_count, cudaStream_t st)
+{
+    dim3 grid(n_pad / 32, n_pad / 32), block(32, 8);
+    prepare_w_kernel<<<grid, block, 0, st>>>(W_in, n, n_pad, Wz, diag, asym_count);
+    return (int)cudaGetLastError();
+}
+
+int launch_zero_start(const Instance &I, SearchState &S, int32_t s0, int32_t s1, cudaStream_t st)
+{
+    if (s1 <= s0) return 0;
+    zero_start_kernel<<<s1 - s0, I.nt, 0, st>>>(I.n, I.nt, I.diag, S.g, S.X, S.B, S.E, S.EB, S.a, S.hash, S.flips,
+                                                 S.sflips, s0);
+    return (int)cudaGetLastError();
+}
+
+int launch_batch_init(const Instance &I, const uint8_t *X, int32_t count, int64_t *E, int32_t *delta,
+                      cudaStream_t st)
+{
+    if (count <= 0) return 0;
+    cudaMemsetAsync(E, 0, sizeof(int64_t) * (size_t)count, st);
+    dim3 grid(I.n_pad / kInitT, (count + kInitB - 1) / kInitB);
+    const size_t smem = (size_t)kInitB * (I.n_pad / 32) * sizeof(uint32_t);
+    cudaFuncSetAttribute(batch_init_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    batch_init_kernel<<<grid, kInitT, smem, st>>>(I.Wz, I.diag, I.n, I.n_pad, X, count, E, delta);
+    return (int)cudaGetLastError();
+}
+
+}  // namespace absb
