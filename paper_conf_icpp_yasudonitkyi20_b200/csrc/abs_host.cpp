@@ -161,6 +161,7 @@ static void free_ctx(abs_ctx *c)
     if (c->st) cudaStreamSynchronize(c->st);
     cudaFree(c->I.Wz);
     cudaFree(c->I.diag);
+    cudaFree(c->I.rowmax);
     cudaFree(c->S.g);
     cudaFree(c->S.X);
     cudaFree(c->S.B);
@@ -283,6 +284,7 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
     c->bytes_per_vec = I.n_pad / 8;
     CTX_CU(cudaMalloc(&I.Wz, (size_t)I.n_pad * I.n_pad * sizeof(int16_t)));
     CTX_CU(cudaMalloc(&I.diag, (size_t)I.n_pad * sizeof(int32_t)));
+    CTX_CU(cudaMalloc(&I.rowmax, (size_t)I.n_pad * sizeof(int32_t)));
     {
         int16_t *W_in = nullptr;
         const size_t wbytes = (size_t)n * n * sizeof(int16_t);
@@ -307,6 +309,9 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
         CTX_CU(e2);
         CTX_CU(e3);
         if (bad) return bail(fail(ABS_EINVAL, "W is not symmetric (" + std::to_string(bad) + " entries)"));
+        const int rc2 = launch_rowmax(I, c->st);
+        c->launches++;
+        if (rc2) return bail(fail(ABS_ECUDA, std::string("rowmax: ") + cudaGetErrorString((cudaError_t)rc2)));
     }
 
     // ---- per-search state
@@ -364,6 +369,7 @@ static int lockstep_step(abs_ctx *c)
     c->h2d += (int64_t)S * bpv;
     RoundArgs a{};
     a.Wz = c->I.Wz;
+    a.rowmax = c->I.rowmax;
     a.n = c->I.n;
     a.n_pad = c->I.n_pad;
     a.nt = c->I.nt;

@@ -23,6 +23,7 @@ struct Instance {
     int32_t n = 0, n_pad = 0, nt = 0;
     int16_t *Wz = nullptr;
     int32_t *diag = nullptr;
+    int32_t *rowmax = nullptr;  // [n_pad] max_i |W_ik| (i != k): bound on one flip's change of any Delta
 };
 
 // Per-search state, structure of arrays (index = local search id).
@@ -41,6 +42,7 @@ struct SearchState {
 
 struct RoundArgs {
     const int16_t *Wz;
+    const int32_t *rowmax;
     int32_t n, n_pad, nt;
     int32_t *g;
     uint8_t *X;
@@ -58,6 +60,7 @@ struct RoundArgs {
 // Launchers (return cudaError_t as int).
 int launch_prepare_w(const int16_t *W_in, int32_t n, int32_t n_pad, int16_t *Wz, int32_t *diag,
                      unsigned long long *asym_count, cudaStream_t st);
+int launch_rowmax(const Instance &I, cudaStream_t st);
 int launch_zero_start(const Instance &I, SearchState &S, int32_t s0, int32_t s1, cudaStream_t st);
 int launch_round(const RoundArgs &a, cudaStream_t st);
 // Batched init: X bytes [count][n_pad/8] -> E [count], and either

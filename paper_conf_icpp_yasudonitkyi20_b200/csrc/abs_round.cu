@@ -146,15 +146,25 @@ __device__ __forceinline__ int lowest_equal(const int (&g)[32], uint32_t xm, uin
 {
     int r = INT_MAX;
 #pragma unroll
-    for (int s = 31; s >= 0; --s)
-        if (((cm >> s) & 1u) && readout(g[s], xm, s) == v) r = 2 * slot_index(t, nt, s) + (int)((xm >> s) & 1u);
+    for (int s = 0; s < 32; ++s) {
+        const bool hit = ((cm >> s) & 1u) && readout(g[s], xm, s) == v;
+        if (hit && r == INT_MAX) r = 2 * slot_index(t, nt, s) + (int)((xm >> s) & 1u);
+    }
     return r;
 }
 
-// Row update for one flip: g += c * W_k* over the 32 slots, then the n
-// neighbour deltas (Eq.(5)) -> min over all (vmin) and, kStraight, min over
-// the mismatch set (cmin).
-template <bool kStraight>
+// Byte-group j (0..3) of bit i: i >> 3 = t + nt*j with t < nt (no division).
+__device__ __forceinline__ int group_of(int i, int nt)
+{
+    const int beta = i >> 3;
+    return (beta >= nt) + (beta >= 2 * nt) + (beta >= 3 * nt);
+}
+
+// Row update for one flip: g += c * W_k* over the 32 slots (Eq.(16), field
+// form), then, unless kMode == kUpdate, the n neighbour deltas (Eq.(5)):
+// min over all bits (vmin) and, kMode == kStraight, over the mismatches (cmin).
+enum { kUpdate = 0, kMin = 1, kStraight = 2 };
+template <int kMode>
 __device__ __forceinline__ void process_row(int (&g)[32], uint32_t xm, uint32_t mism, const uint4 *row4,
                                             uint64_t *bars, uint32_t par, int c, int t, int nt, int &vmin,
                                             int &cmin)
@@ -169,15 +179,17 @@ __device__ __forceinline__ void process_row(int (&g)[32], uint32_t xm, uint32_t 
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
             const int s0 = 8 * j + 2 * q;
-            g[s0] += c * sext16(wv[q]);         // Eq.(16), field form
+            g[s0] += c * sext16(wv[q]);
             g[s0 + 1] += c * (((int)wv[q]) >> 16);
-            const int d0 = readout(g[s0], xm, s0);
-            const int d1 = readout(g[s0 + 1], xm, s0 + 1);
-            vmin = min(vmin, min(d0, d1));
-            if (kStraight) {
-                const int m0 = ((mism >> s0) & 1u) ? d0 : INT_MAX;
-                const int m1 = ((mism >> (s0 + 1)) & 1u) ? d1 : INT_MAX;
-                cmin = min(cmin, min(m0, m1));
+            if (kMode != kUpdate) {
+                const int d0 = readout(g[s0], xm, s0);
+                const int d1 = readout(g[s0 + 1], xm, s0 + 1);
+                vmin = min(vmin, min(d0, d1));
+                if (kMode == kStraight) {
+                    const int m0 = ((mism >> s0) & 1u) ? d0 : INT_MAX;
+                    const int m1 = ((mism >> (s0 + 1)) & 1u) ? d1 : INT_MAX;
+                    cmin = min(cmin, min(m0, m1));
+                }
             }
         }
     }
@@ -187,7 +199,7 @@ __device__ __forceinline__ void process_row(int (&g)[32], uint32_t xm, uint32_t 
 struct RoundSmem {
     uint64_t bar[2][4];   // [row buffer][chunk]
     Red red[2][32];
-    int sel[2][3];        // window warp -> all: next (k, Delta_k, x_k), by flip parity
+    int sel[2][4];        // window warp -> all: next (k, Delta_k, x_k, rowmax_k), by flip parity
     uint64_t hash;        // thread 0 only
     long long nflip, nstraight;
 };
@@ -211,14 +223,16 @@ __device__ __forceinline__ void issue_row(const RoundArgs &A, int k, unsigned ch
 __device__ __forceinline__ void publish_window(const int (&g)[32], uint32_t xm, int a2, int l, int n, int t, int nt,
                                                int *wd, uint8_t *wx)
 {
+    // window bytes: [b0, b1] and, when the window wraps (reading C6), [0, b2]
     const int end = a2 + l;
-    const int hi1 = min(end, n);
-    const int hi2 = end - n;
+    const int b0 = a2 >> 3;
+    const int b1 = (min(end, n) - 1) >> 3;
+    const int b2 = end > n ? ((end - n - 1) >> 3) : -1;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-        const int base = 8 * (t + nt * j);
-        const bool hit = ((base + 8 > a2) && (base < hi1)) || (base < hi2);
-        if (hit) {
+        const int beta = t + nt * j;
+        if ((unsigned)(beta - b0) <= (unsigned)(b1 - b0) || beta <= b2) {
+            const int base = 8 * beta;
 #pragma unroll
             for (int e = 0; e < 8; ++e) {
                 const int i = base + e;
@@ -291,9 +305,16 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
     if (kMulti) __syncthreads();
     else __syncwarp();
 
+    // Lower bound on min_i Delta_i(X) for the lazy neighbour tracking of the
+    // prefetch path: exact after every CTA reduction; after flipping k,
+    //   min_i Delta_i(X') >= min(LB - 2*rowmax_k, -Delta_k(X))     (Eq.(16), Eq.(6)),
+    // and if E(X') + min(0, LB) >= E_B no neighbour of X' can improve B, so
+    // the n readouts of that flip can be skipped without changing any result.
+    int64_t LB = INT64_MIN / 4;
+
     // ---- first selection of the round
     bool straight = block_any<kMulti>(xm != stm[t]);
-    int k, dk, xk;
+    int k, dk, xk, rk = 32768;  // rk: rowmax of k (|W| <= 32768 before it is known)
     {
         int cv, ci2;
         const uint32_t cm = straight ? (xm ^ stm[t]) : window_mask(a, l, n, t, nt);
@@ -319,6 +340,17 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
         if (pre && !straight && left > 1 && warp == 0) {
             int a1 = a + l;
             if (a1 >= n) a1 -= n;
+            {
+                // wait for the chunks of row k_f that hold the window's bits
+                const int end = a1 + l - 1;
+                const int c0 = group_of(a1, nt);
+                const int c1 = group_of(min(end, n - 1), nt);
+                for (int cc = c0; cc <= c1; ++cc) mbar_wait(&sm->bar[b][cc], par);
+                if (end >= n) {
+                    const int c2 = group_of(end - n, nt);
+                    for (int cc = 0; cc <= c2; ++cc) mbar_wait(&sm->bar[b][cc], par);
+                }
+            }
             const int *wd = win->d[b];
             const uint8_t *wx = win->x[b];
             const short *rw = reinterpret_cast<const short *>(row);
@@ -326,12 +358,11 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
             for (int r = lane; r < l; r += 32) {
                 int i = a1 + r;
                 if (i >= n) i -= n;
-                mbar_wait(&sm->bar[b][(i >> 3) / nt], par);
                 const int xi = wx[r];
                 int d = wd[r];
                 int xn = xi;
                 if (i == k) {
-                    d = -d;      // Eq.(6), k = i
+                    d = -d;  // Eq.(6), k = i
                     xn ^= 1;
                 } else {
                     const int w2 = 2 * (int)rw[i];
@@ -346,10 +377,11 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
             const int mv = __reduce_min_sync(kFull, bv);
             const int mi = __reduce_min_sync(kFull, bv == mv ? 2 * bi + bx : INT_MAX);
             if (lane == 0) {
+                issue_row(A, mi >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
                 sm->sel[b][0] = mi >> 1;
                 sm->sel[b][1] = mv;
                 sm->sel[b][2] = mi & 1;
-                issue_row(A, mi >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+                sm->sel[b][3] = __ldg(A.rowmax + (mi >> 1));
             }
         }
 
@@ -362,17 +394,23 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
         const int c = xk ? -2 : 2;  // 2 phi(x_k), pre-flip bit (Eq.(16))
         E += dk;                    // E(X) <- E(X) + d_k
         {
-            const int beta = k >> 3;
-            if (t == beta % nt) xm ^= 1u << (8 * (beta / nt) + (k & 7));  // x_k <- 1 - x_k
+            const int j = group_of(k, nt);
+            if (t == (k >> 3) - nt * j) xm ^= 1u << (8 * j + (k & 7));  // x_k <- 1 - x_k
+        }
+        bool exact = true;
+        if (pre && !straight) {
+            LB = min(LB - 2 * (int64_t)rk, -(int64_t)dk);
+            exact = E + min(LB, (int64_t)0) < EB;  // uniform
         }
         int vmin, cmin;
         const uint4 *row4 = reinterpret_cast<const uint4 *>(row);
         uint32_t mism = 0;
         if (straight) {
             mism = xm ^ stm[t];
-            process_row<true>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
+            process_row<kStraight>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
         } else {
-            process_row<false>(g, xm, 0u, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
+            if (exact) process_row<kMin>(g, xm, 0u, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
+            else process_row<kUpdate>(g, xm, 0u, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
             a += l;  // offset <- (a + l) mod n
             if (a >= n) a -= n;
         }
@@ -387,11 +425,18 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
                 if (__any_sync(kFull, cm != 0u)) candidates(g, xm, cm, t, nt, cmin, ci2);
             }
         }
-        const Red r1 = block_reduce<kMulti>(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw);
+        Red r1;
+        if (exact) {
+            r1 = block_reduce<kMulti>(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw);
+            LB = r1.v;
+        } else {
+            __syncthreads();  // row buffer b free, sel[b] and the window published
+            r1 = Red{INT_MAX, INT_MAX, INT_MAX};
+        }
 
         // ---- neighbour tracking (reading C2) and, straight phase, the argmin index
         const int64_t cand = E + (r1.v < 0 ? (int64_t)r1.v : 0);
-        const bool improve = cand < EB;  // uniform
+        const bool improve = exact && cand < EB;  // uniform
         const bool sidx = straight && r1.c != INT_MAX;
         if (improve || sidx) {
             int it = INT_MAX, is = INT_MAX;
@@ -402,8 +447,8 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
                 uint32_t bm = xm;
                 if (r1.v < 0) {
                     const int istar = r2.v >> 1;
-                    const int beta = istar >> 3;
-                    if (t == beta % nt) bm ^= 1u << (8 * (beta / nt) + (istar & 7));
+                    const int j = group_of(istar, nt);
+                    if (t == (istar >> 3) - nt * j) bm ^= 1u << (8 * j + (istar & 7));
                 }
                 sbm[t] = bm;
                 EB = cand;
@@ -422,6 +467,7 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
                 k = sm->sel[b][0];
                 dk = sm->sel[b][1];
                 xk = sm->sel[b][2];
+                rk = sm->sel[b][3];
                 continue;  // row already in flight
             }
             k = r1.i >> 1;
@@ -442,6 +488,7 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
             k = r.i >> 1;
             xk = r.i & 1;
             dk = r.c;
+            rk = __ldg(A.rowmax + k);
         }
         if (t == 0) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
     }

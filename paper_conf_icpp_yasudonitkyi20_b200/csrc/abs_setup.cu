@@ -46,6 +46,24 @@ __global__ void prepare_w_kernel(const int16_t *__restrict__ W, int n, int n_pad
     if (bad) atomicAdd(asym, bad);
 }
 
+// rowmax[k] = max_i |Wz_ik|: every Delta_i (i != k) moves by at most 2*rowmax[k]
+// when bit k flips (Eq.(16)); used by the round kernel's lazy minimum.
+__global__ void rowmax_kernel(const int16_t *__restrict__ Wz, int n_pad, int32_t *__restrict__ rowmax)
+{
+    __shared__ int red[32];
+    const int k = blockIdx.x;
+    int m = 0;
+    for (int i = threadIdx.x; i < n_pad; i += blockDim.x) m = max(m, abs((int)Wz[(size_t)k * n_pad + i]));
+    m = __reduce_max_sync(kFull, m);
+    if ((threadIdx.x & 31) == 0) red[threadIdx.x >> 5] = m;
+    __syncthreads();
+    if (threadIdx.x < 32) {
+        m = threadIdx.x < (int)(blockDim.x >> 5) ? red[threadIdx.x] : 0;
+        m = __reduce_max_sync(kFull, m);
+        if (threadIdx.x == 0) rowmax[k] = m;
+    }
+}
+
 // Device Step 1: C = 0, E = 0, Delta_i = W_ii (g_i = W_ii).
 __global__ void zero_start_kernel(int n, int nt, const int32_t *__restrict__ diag, int32_t *g, uint8_t *X,
                                   uint8_t *B, int64_t *E, int64_t *EB, int32_t *a, uint64_t *hash, int64_t *flips,
@@ -146,6 +164,12 @@ int launch_prepare_w(const int16_t *W_in, int32_t n, int32_t n_pad, int16_t *Wz,
 {
     dim3 grid(n_pad / 32, n_pad / 32), block(32, 8);
     prepare_w_kernel<<<grid, block, 0, st>>>(W_in, n, n_pad, Wz, diag, asym_count);
+    return (int)cudaGetLastError();
+}
+
+int launch_rowmax(const Instance &I, cudaStream_t st)
+{
+    rowmax_kernel<<<I.n_pad, 256, 0, st>>>(I.Wz, I.n_pad, I.rowmax);
     return (int)cudaGetLastError();
 }
 
