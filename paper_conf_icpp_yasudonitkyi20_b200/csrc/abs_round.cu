@@ -98,7 +98,10 @@ __device__ __forceinline__ Red block_reduce(Red r, Red (*sred)[32], int &rb, int
     w.v = __reduce_min_sync(kFull, r.v);
     w.c = __reduce_min_sync(kFull, r.c);
     w.i = __reduce_min_sync(kFull, r.c == w.c ? r.i : INT_MAX);
-    if (!kMulti) return w;
+    if (!kMulti) {
+        __syncwarp();  // orders lane 0's shared-memory bookkeeping before the other lanes read it
+        return w;
+    }
     Red *buf = sred[rb & 1];
     ++rb;
     if (lane == 0) buf[warp] = w;
@@ -122,6 +125,29 @@ __device__ __forceinline__ bool block_any(bool p)
 {
     if (!kMulti) return __any_sync(kFull, p);
     return __syncthreads_or(p) != 0;
+}
+
+// Register pressure: in the 1024-thread kernel, slots 24..31 (byte-group 3)
+// live in shared memory between uses ([2][nt] int4, conflict-free).  Volatile
+// PTX so the compiler cannot forward the stored values and keep them live.
+__device__ __forceinline__ void hi_load(int (&g)[32], const int4 *sgh, int t, int nt)
+{
+    asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(g[24]), "=r"(g[25]), "=r"(g[26]), "=r"(g[27])
+                 : "r"(smem_u32(sgh + t)));
+    asm volatile("ld.shared.v4.s32 {%0, %1, %2, %3}, [%4];"
+                 : "=r"(g[28]), "=r"(g[29]), "=r"(g[30]), "=r"(g[31])
+                 : "r"(smem_u32(sgh + nt + t)));
+}
+
+__device__ __forceinline__ void hi_store(const int (&g)[32], int4 *sgh, int t, int nt)
+{
+    asm volatile("st.shared.v4.s32 [%0], {%1, %2, %3, %4};" ::"r"(smem_u32(sgh + t)), "r"(g[24]), "r"(g[25]),
+                 "r"(g[26]), "r"(g[27])
+                 : "memory");
+    asm volatile("st.shared.v4.s32 [%0], {%1, %2, %3, %4};" ::"r"(smem_u32(sgh + nt + t)), "r"(g[28]), "r"(g[29]),
+                 "r"(g[30]), "r"(g[31])
+                 : "memory");
 }
 
 // Lowest-index argmin over the slots in `cm`; ci2 = 2*index + x (INT_MAX if none).
@@ -164,15 +190,16 @@ __device__ __forceinline__ int group_of(int i, int nt)
 // form), then, unless kMode == kUpdate, the n neighbour deltas (Eq.(5)):
 // min over all bits (vmin) and, kMode == kStraight, over the mismatches (cmin).
 enum { kUpdate = 0, kMin = 1, kStraight = 2 };
-template <int kMode>
+template <int kMode, bool kHi>
 __device__ __forceinline__ void process_row(int (&g)[32], uint32_t xm, uint32_t mism, const uint4 *row4,
                                             uint64_t *bars, uint32_t par, int c, int t, int nt, int &vmin,
-                                            int &cmin)
+                                            int &cmin, int4 *sgh)
 {
     vmin = INT_MAX;
     cmin = INT_MAX;
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
+        if (kHi && j == 3) hi_load(g, sgh, t, nt);
         mbar_wait(&bars[j], par);
         const uint4 w4 = row4[t + nt * j];
         const uint32_t wv[4] = {w4.x, w4.y, w4.z, w4.w};
@@ -192,6 +219,7 @@ __device__ __forceinline__ void process_row(int (&g)[32], uint32_t xm, uint32_t 
                 }
             }
         }
+        if (kHi && j == 3) hi_store(g, sgh, t, nt);
     }
 }
 
@@ -199,7 +227,9 @@ __device__ __forceinline__ void process_row(int (&g)[32], uint32_t xm, uint32_t 
 struct RoundSmem {
     uint64_t bar[2][4];   // [row buffer][chunk]
     Red red[2][32];
-    int sel[2][4];        // window warp -> all: next (k, Delta_k, x_k, rowmax_k), by flip parity
+    int sel[2][4];        // window warp -> all: next (k, Delta_k, x_k, exact_next), by flip parity
+    int thr[2];           // improvement threshold min(E_B - E(X'), ...) clamped to int32, by flip parity
+    long long E, EB, LB;  // E(X), E_B, lower bound on min_i Delta_i(X): thread 0 only
     uint64_t hash;        // thread 0 only
     long long nflip, nstraight;
 };
@@ -220,8 +250,8 @@ __device__ __forceinline__ void issue_row(const RoundArgs &A, int k, unsigned ch
 }
 
 // Owners of the bits of window {(a2 + r) mod n : r < l} publish Delta and x.
-__device__ __forceinline__ void publish_window(const int (&g)[32], uint32_t xm, int a2, int l, int n, int t, int nt,
-                                               int *wd, uint8_t *wx)
+__device__ __forceinline__ void publish_window(int (&g)[32], uint32_t xm, int a2, int l, int n, int t, int nt,
+                                               int *wd, uint8_t *wx, const int4 *sgh)
 {
     // window bytes: [b0, b1] and, when the window wraps (reading C6), [0, b2]
     const int end = a2 + l;
@@ -232,6 +262,7 @@ __device__ __forceinline__ void publish_window(const int (&g)[32], uint32_t xm, 
     for (int j = 0; j < 4; ++j) {
         const int beta = t + nt * j;
         if ((unsigned)(beta - b0) <= (unsigned)(b1 - b0) || beta <= b2) {
+            if (j == 3 && sgh) hi_load(g, sgh, t, nt);
             const int base = 8 * beta;
 #pragma unroll
             for (int e = 0; e < 8; ++e) {
@@ -247,11 +278,11 @@ __device__ __forceinline__ void publish_window(const int (&g)[32], uint32_t xm, 
     }
 }
 
-template <bool kMulti>
+template <bool kMulti, int kNT>
 __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_kernel(const RoundArgs A)
 {
     extern __shared__ __align__(128) unsigned char smem[];
-    const int nt = kMulti ? A.nt : 32;
+    const int nt = kNT ? kNT : (kMulti ? A.nt : 32);  // compile-time for the common sizes
     const int n = A.n;
     const int t = threadIdx.x;
     const int lane = t & 31, warp = t >> 5, nw = nt >> 5;
@@ -263,6 +294,7 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
     uint32_t *stm = reinterpret_cast<uint32_t *>(smem + 2 * rowb + sizeof(RoundSmem));  // [nt] target bits
     uint32_t *sbm = stm + nt;                                                          // [nt] best bits
     WindowSmem *win = reinterpret_cast<WindowSmem *>(sbm + nt);                         // kMulti only
+    int4 *sgh = reinterpret_cast<int4 *>((reinterpret_cast<uintptr_t>(win + 1) + 15) & ~uintptr_t(15));  // [2][nt]
 
     if (t == 0) {
 #pragma unroll
@@ -273,6 +305,15 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
         sm->hash = A.hash[sid];
         sm->nflip = 0;
         sm->nstraight = 0;
+        sm->E = A.E[sid];
+        sm->EB = sm->E;  // Step 3, reading C4: E_B = E(C) (Alg. 5) ...
+        // Lower bound on min_i Delta_i(X) (lazy neighbour tracking, prefetch
+        // path): after flipping k, min_i Delta_i(X') >= min(LB - 2*rowmax_k,
+        // -Delta_k(X)) (Eq.(16), Eq.(6)); if E(X') + min(0, LB) >= E_B no
+        // neighbour of X' can improve B and the n readouts may be skipped
+        // without changing any result.  Tightened to the exact minimum after
+        // every CTA reduction.
+        sm->LB = INT64_MIN / 4;
     }
 
     // ---- load the search state (registers for the whole round)
@@ -281,6 +322,7 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
         const int32_t *gs = A.g + (size_t)sid * 32 * nt;
 #pragma unroll
         for (int s = 0; s < 32; ++s) g[s] = gs[(size_t)s * nt + t];
+        if (kMulti) hi_store(g, sgh, t, nt);
     }
     uint32_t xm = 0;
     {
@@ -293,10 +335,8 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
             tm |= (uint32_t)Ts[t + nt * j] << (8 * j);  // Step 2: read target T
         }
         stm[t] = tm;
-        sbm[t] = xm;  // Step 3, reading C4: B = C ...
+        sbm[t] = xm;  // ... and B = C
     }
-    int64_t E = A.E[sid];
-    int64_t EB = E;  // ... and E_B = E(C) (Alg. 5)
     int a = A.a[sid];
     const int l = A.l[sid];
     const bool pre = kMulti && l <= kWinMax;
@@ -305,31 +345,30 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
     if (kMulti) __syncthreads();
     else __syncwarp();
 
-    // Lower bound on min_i Delta_i(X) for the lazy neighbour tracking of the
-    // prefetch path: exact after every CTA reduction; after flipping k,
-    //   min_i Delta_i(X') >= min(LB - 2*rowmax_k, -Delta_k(X))     (Eq.(16), Eq.(6)),
-    // and if E(X') + min(0, LB) >= E_B no neighbour of X' can improve B, so
-    // the n readouts of that flip can be skipped without changing any result.
-    int64_t LB = INT64_MIN / 4;
-
     // ---- first selection of the round
     bool straight = block_any<kMulti>(xm != stm[t]);
-    int k, dk, xk, rk = 32768;  // rk: rowmax of k (|W| <= 32768 before it is known)
+    int k, dk, xk;
     {
         int cv, ci2;
         const uint32_t cm = straight ? (xm ^ stm[t]) : window_mask(a, l, n, t, nt);
+        if (kMulti) hi_load(g, sgh, t, nt);
         candidates(g, xm, cm, t, nt, cv, ci2);
         if (pre && !straight) {
             int a2 = a + l;
             if (a2 >= n) a2 -= n;
-            publish_window(g, xm, a2, l, n, t, nt, win->d[0], win->x[0]);
+            publish_window(g, xm, a2, l, n, t, nt, win->d[0], win->x[0], sgh);
         }
         const Red r = block_reduce<kMulti>(Red{INT_MAX, cv, ci2}, sm->red, rb, lane, warp, nw);
         k = r.i >> 1;
         xk = r.i & 1;
         dk = r.c;
     }
-    if (t == 0) issue_row(A, k, rowbuf, sm->bar[0], nt);
+    bool exact = true;  // compute the n neighbour deltas of this flip exactly
+    int rk = 0;         // thread 0: rowmax of the row being flipped
+    if (t == 0) {
+        rk = __ldg(A.rowmax + k);
+        issue_row(A, k, rowbuf, sm->bar[0], nt);
+    }
 
     for (int f = 0;; ++f) {
         const int b = f & 1;
@@ -337,6 +376,7 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
         unsigned char *row = rowbuf + rowb * b;
 
         // ---- window-first selection of the next flip (warp 0), prefetch its row
+        int rk_next = 0;
         if (pre && !straight && left > 1 && warp == 0) {
             int a1 = a + l;
             if (a1 >= n) a1 -= n;
@@ -355,23 +395,43 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
             const uint8_t *wx = win->x[b];
             const short *rw = reinterpret_cast<const short *>(row);
             int bv = INT_MAX, bi = INT_MAX, bx = 0;
-            for (int r = lane; r < l; r += 32) {
-                int i = a1 + r;
-                if (i >= n) i -= n;
-                const int xi = wx[r];
-                int d = wd[r];
-                int xn = xi;
-                if (i == k) {
-                    d = -d;  // Eq.(6), k = i
-                    xn ^= 1;
-                } else {
-                    const int w2 = 2 * (int)rw[i];
-                    d += (xi == xk) ? w2 : -w2;  // Eq.(16)
+            // l <= kWinMax = 8 * 32: a lane's loads are issued in two batches of four
+#pragma unroll
+            for (int h = 0; h < kWinMax / 128; ++h) {
+                int dd[4], ww[4], xx[4], ii[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int r = lane + 32 * (4 * h + q);
+                    int i = a1 + r;
+                    if (i >= n) i -= n;
+                    ii[q] = i;
+                    dd[q] = 0;
+                    xx[q] = 0;
+                    ww[q] = 0;
+                    if (r < l) {
+                        dd[q] = wd[r];
+                        xx[q] = wx[r];
+                        ww[q] = rw[i];
+                    }
                 }
-                if (d < bv || (d == bv && i < bi)) {
-                    bv = d;
-                    bi = i;
-                    bx = xn;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    if (lane + 32 * (4 * h + q) < l) {
+                        const int i = ii[q];
+                        int d = dd[q];
+                        int xn = xx[q];
+                        if (i == k) {
+                            d = -d;  // Eq.(6), k = i
+                            xn ^= 1;
+                        } else {
+                            d += (xx[q] == xk) ? 2 * ww[q] : -2 * ww[q];  // Eq.(16)
+                        }
+                        if (d < bv || (d == bv && i < bi)) {
+                            bv = d;
+                            bi = i;
+                            bx = xn;
+                        }
+                    }
                 }
             }
             const int mv = __reduce_min_sync(kFull, bv);
@@ -381,36 +441,25 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
                 sm->sel[b][0] = mi >> 1;
                 sm->sel[b][1] = mv;
                 sm->sel[b][2] = mi & 1;
-                sm->sel[b][3] = __ldg(A.rowmax + (mi >> 1));
+                rk_next = __ldg(A.rowmax + (mi >> 1));  // consumed after the row update
             }
         }
 
         // ---- flip k (Alg. 4 lines P:L328-336 / Alg. 5 lines P:L371-376)
-        if (t == 0) {
-            sm->hash = (sm->hash ^ (uint64_t)(uint32_t)k) * kFnvPrime;
-            sm->nflip += 1;
-            if (straight) sm->nstraight += 1;
-        }
         const int c = xk ? -2 : 2;  // 2 phi(x_k), pre-flip bit (Eq.(16))
-        E += dk;                    // E(X) <- E(X) + d_k
         {
             const int j = group_of(k, nt);
             if (t == (k >> 3) - nt * j) xm ^= 1u << (8 * j + (k & 7));  // x_k <- 1 - x_k
-        }
-        bool exact = true;
-        if (pre && !straight) {
-            LB = min(LB - 2 * (int64_t)rk, -(int64_t)dk);
-            exact = E + min(LB, (int64_t)0) < EB;  // uniform
         }
         int vmin, cmin;
         const uint4 *row4 = reinterpret_cast<const uint4 *>(row);
         uint32_t mism = 0;
         if (straight) {
             mism = xm ^ stm[t];
-            process_row<kStraight>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
+            process_row<kStraight, kMulti>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, cmin, sgh);
         } else {
-            if (exact) process_row<kMin>(g, xm, 0u, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
-            else process_row<kUpdate>(g, xm, 0u, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
+            if (exact) process_row<kMin, kMulti>(g, xm, 0u, row4, sm->bar[b], par, c, t, nt, vmin, cmin, sgh);
+            else process_row<kUpdate, kMulti>(g, xm, 0u, row4, sm->bar[b], par, c, t, nt, vmin, cmin, sgh);
             a += l;  // offset <- (a + l) mod n
             if (a >= n) a -= n;
         }
@@ -419,27 +468,55 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
             if (pre) {
                 int a2 = a + l;
                 if (a2 >= n) a2 -= n;
-                publish_window(g, xm, a2, l, n, t, nt, win->d[b ^ 1], win->x[b ^ 1]);
+                publish_window(g, xm, a2, l, n, t, nt, win->d[b ^ 1], win->x[b ^ 1], sgh);
             } else {
                 const uint32_t cm = window_mask(a, l, n, t, nt);
-                if (__any_sync(kFull, cm != 0u)) candidates(g, xm, cm, t, nt, cmin, ci2);
+                if (__any_sync(kFull, cm != 0u)) {
+                    if (kMulti) hi_load(g, sgh, t, nt);
+                    candidates(g, xm, cm, t, nt, cmin, ci2);
+                }
+            }
+        }
+        // ---- thread 0: E(X') = E(X) + d_k, the bound LB, the improvement
+        // threshold, and (prefetch path) whether the next flip must be exact
+        if (t == 0) {
+            sm->hash = (sm->hash ^ (uint64_t)(uint32_t)k) * kFnvPrime;
+            sm->nflip += 1;
+            if (straight) sm->nstraight += 1;
+            const long long E1 = sm->E + dk;
+            const long long LB1 = min(sm->LB - 2 * (long long)rk, -(long long)dk);
+            const long long EB = sm->EB;
+            sm->E = E1;
+            sm->LB = LB1;
+            // cand = E(X') + min(0, m) < E_B  <=>  min(0, m) < E_B - E(X')   (<= 2^31 - 32768
+            // because E_B <= E(X); clamped below at INT_MIN, where it can never hold)
+            sm->thr[b] = (int)max(EB - E1, (long long)INT_MIN);
+            if (pre && !straight && left > 1) {
+                // E_B may still drop in this flip: the current (larger) E_B only makes
+                // the test more conservative
+                const int dk1 = sm->sel[b][1];
+                const long long LB2 = min(LB1 - 2 * (long long)rk_next, -(long long)dk1);
+                sm->sel[b][3] = (E1 + dk1 + min(LB2, 0LL) < EB) ? 1 : 0;
             }
         }
         Red r1;
         if (exact) {
             r1 = block_reduce<kMulti>(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw);
-            LB = r1.v;
         } else {
-            __syncthreads();  // row buffer b free, sel[b] and the window published
+            __syncthreads();  // row buffer b free; sel[b], thr[b] and the window published
             r1 = Red{INT_MAX, INT_MAX, INT_MAX};
         }
 
         // ---- neighbour tracking (reading C2) and, straight phase, the argmin index
-        const int64_t cand = E + (r1.v < 0 ? (int64_t)r1.v : 0);
-        const bool improve = exact && cand < EB;  // uniform
+        const bool improve = exact && min(r1.v, 0) < sm->thr[b];  // uniform
+        if (t == 0 && exact) {
+            sm->LB = r1.v;
+            if (improve) sm->EB = sm->E + min(r1.v, 0);
+        }
         const bool sidx = straight && r1.c != INT_MAX;
         if (improve || sidx) {
             int it = INT_MAX, is = INT_MAX;
+            if (kMulti) hi_load(g, sgh, t, nt);
             if (improve && r1.v < 0 && vmin == r1.v) it = lowest_equal(g, xm, 0xffffffffu, r1.v, t, nt);
             if (sidx && cmin == r1.c) is = lowest_equal(g, xm, mism, r1.c, t, nt);
             const Red r2 = block_reduce<kMulti>(Red{it, is, is}, sm->red, rb, lane, warp, nw);
@@ -451,7 +528,6 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
                     if (t == (istar >> 3) - nt * j) bm ^= 1u << (8 * j + (istar & 7));
                 }
                 sbm[t] = bm;
-                EB = cand;
             }
             if (sidx) {
                 k = r2.c >> 1;
@@ -467,7 +543,8 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
                 k = sm->sel[b][0];
                 dk = sm->sel[b][1];
                 xk = sm->sel[b][2];
-                rk = sm->sel[b][3];
+                exact = sm->sel[b][3] != 0;
+                rk = rk_next;
                 continue;  // row already in flight
             }
             k = r1.i >> 1;
@@ -478,24 +555,30 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
             straight = false;
             if (left <= 0) break;
             int cv, cj;
+            if (kMulti) hi_load(g, sgh, t, nt);
             candidates(g, xm, window_mask(a, l, n, t, nt), t, nt, cv, cj);
             if (pre) {
                 int a2 = a + l;
                 if (a2 >= n) a2 -= n;
-                publish_window(g, xm, a2, l, n, t, nt, win->d[b ^ 1], win->x[b ^ 1]);
+                publish_window(g, xm, a2, l, n, t, nt, win->d[b ^ 1], win->x[b ^ 1], sgh);
             }
             const Red r = block_reduce<kMulti>(Red{INT_MAX, cv, cj}, sm->red, rb, lane, warp, nw);
             k = r.i >> 1;
             xk = r.i & 1;
             dk = r.c;
-            rk = __ldg(A.rowmax + k);
+            exact = true;
         }
-        if (t == 0) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+        if (t == 0) {
+            rk = __ldg(A.rowmax + k);
+            issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+        }
     }
 
     // ---- Step 5: store (B, E_B) and the state C' for the next round
     if (kMulti) __syncthreads();
+    else __syncwarp();
     {
+        if (kMulti) hi_load(g, sgh, t, nt);
         int32_t *gs = A.g + (size_t)sid * 32 * nt;
 #pragma unroll
         for (int s = 0; s < 32; ++s) gs[(size_t)s * nt + t] = g[s];
@@ -508,8 +591,8 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
             Bs[t + nt * j] = (uint8_t)(bm >> (8 * j));
         }
         if (t == 0) {
-            A.E[sid] = E;
-            A.EB[sid] = EB;
+            A.E[sid] = sm->E;
+            A.EB[sid] = sm->EB;
             A.a[sid] = a;
             A.hash[sid] = sm->hash;
             A.flips[sid] += sm->nflip;
@@ -523,7 +606,7 @@ __global__ void __launch_bounds__(kMulti ? 1024 : 32, kMulti ? 1 : 32) round_ker
 size_t round_smem_bytes(int32_t nt)
 {
     size_t s = 2 * (size_t)64 * nt + sizeof(RoundSmem) + 2 * sizeof(uint32_t) * (size_t)nt;
-    if (nt > 32) s += sizeof(WindowSmem);
+    if (nt > 32) s += sizeof(WindowSmem) + 16 + 2 * sizeof(int4) * (size_t)nt;
     return s;
 }
 
@@ -531,11 +614,15 @@ int launch_round(const RoundArgs &a, cudaStream_t st)
 {
     const size_t smem = round_smem_bytes(a.nt);
     if (a.nt == 32) {
-        auto k = round_kernel<false>;
+        auto k = round_kernel<false, 32>;
         cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         k<<<a.S, 32, smem, st>>>(a);
+    } else if (a.nt == 1024) {
+        auto k = round_kernel<true, 1024>;
+        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        k<<<a.S, 1024, smem, st>>>(a);
     } else {
-        auto k = round_kernel<true>;
+        auto k = round_kernel<true, 0>;
         cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         k<<<a.S, a.nt, smem, st>>>(a);
     }
