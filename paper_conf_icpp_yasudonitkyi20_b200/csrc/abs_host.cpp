@@ -279,8 +279,7 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
     // ---- instance layout
     Instance &I = c->I;
     I.n = n;
-    I.n_pad = ((n + 1023) / 1024) * 1024;
-    I.nt = I.n_pad / kBitsPerThread;
+    layout_for(n, I.n_pad, I.bpt, I.nt);
     c->bytes_per_vec = I.n_pad / 8;
     CTX_CU(cudaMalloc(&I.Wz, (size_t)I.n_pad * I.n_pad * sizeof(int16_t)));
     CTX_CU(cudaMalloc(&I.diag, (size_t)I.n_pad * sizeof(int32_t)));
@@ -318,7 +317,7 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
     SearchState &S = c->S;
     S.S = cfg.searches;
     const size_t Sn = (size_t)std::max(1, S.S);
-    CTX_CU(cudaMalloc(&S.g, Sn * 32 * I.nt * sizeof(int32_t)));
+    CTX_CU(cudaMalloc(&S.g, Sn * (size_t)I.n_pad * sizeof(int32_t)));
     CTX_CU(cudaMalloc(&S.X, Sn * c->bytes_per_vec));
     CTX_CU(cudaMalloc(&S.B, Sn * c->bytes_per_vec));
     CTX_CU(cudaMalloc(&S.T, Sn * c->bytes_per_vec));
@@ -373,6 +372,7 @@ static int lockstep_step(abs_ctx *c)
     a.n = c->I.n;
     a.n_pad = c->I.n_pad;
     a.nt = c->I.nt;
+    a.bpt = c->I.bpt;
     a.g = c->S.g;
     a.X = c->S.X;
     a.T = c->S.T;
@@ -632,8 +632,8 @@ int abs_search_state(const abs_ctx *c, int32_t s, uint32_t *X_out, int32_t *delt
     ABS_CU(cudaMemcpy(xb.data(), c->S.X + (size_t)s * bpv, bpv, cudaMemcpyDeviceToHost));
     if (X_out) std::memcpy(X_out, xb.data(), sizeof(uint32_t) * words);
     if (delta_out) {
-        std::vector<int32_t> g((size_t)32 * nt);
-        ABS_CU(cudaMemcpy(g.data(), c->S.g + (size_t)s * 32 * nt, sizeof(int32_t) * g.size(),
+        std::vector<int32_t> g((size_t)c->I.n_pad);
+        ABS_CU(cudaMemcpy(g.data(), c->S.g + (size_t)s * c->I.n_pad, sizeof(int32_t) * g.size(),
                           cudaMemcpyDeviceToHost));
         for (int i = 0; i < n; ++i) {
             const int beta = i >> 3, t = beta % nt, slot = 8 * (beta / nt) + (i & 7);

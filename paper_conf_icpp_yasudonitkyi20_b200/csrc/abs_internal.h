@@ -8,26 +8,37 @@
 
 namespace absb {
 
-// Every search keeps P = 32 bits per thread (one uint32 of x bits per thread)
-// and NT threads per search (a multiple of 32, <= 1024), so n_pad = 32 * NT.
-constexpr int kBitsPerThread = 32;
-constexpr int kMaxThreads = 1024;
+// Every search is held by NT threads (a multiple of 32) with P bits each
+// (P = 32 for n <= 3072, else 64), n_pad = P * NT >= n.  Threads hold their
+// P fields in registers; P = 64 gives 512 threads x 128 registers at n = 32k.
+inline void layout_for(int n, int &n_pad, int &bpt, int &nt)
+{
+    const int p1 = ((n + 1023) / 1024) * 1024;
+    if (p1 <= 3072) {
+        bpt = 32;
+        n_pad = p1;
+    } else {
+        bpt = 64;
+        n_pad = ((n + 2047) / 2048) * 2048;
+    }
+    nt = n_pad / bpt;
+}
 
 // Device layout of one instance:
 //   Wz   int16 [n_pad][n_pad]  W with ZERO diagonal, rows/cols >= n zero
 //   diag int32 [n_pad]         W_ii (0 for i >= n)
 // Element i of a search is owned by thread t = (i >> 3) % NT, slot
-// s = 8 * ((i >> 3) / NT) + (i & 7): thread t holds the 4 byte-groups
-// beta = t + NT * j (j = 0..3) of the bit vector, i.e. bits 8*beta .. 8*beta+7.
+// s = 8 * ((i >> 3) / NT) + (i & 7): thread t holds the P/8 byte-groups
+// beta = t + NT * j (j < P/8) of the bit vector, i.e. bits 8*beta .. 8*beta+7.
 struct Instance {
-    int32_t n = 0, n_pad = 0, nt = 0;
+    int32_t n = 0, n_pad = 0, nt = 0, bpt = 32;
     int16_t *Wz = nullptr;
     int32_t *diag = nullptr;
     int32_t *rowmax = nullptr;  // [n_pad] max_i |W_ik| (i != k): bound on one flip's change of any Delta
 };
 
 // Per-search state, structure of arrays (index = local search id).
-//   g     int32 [S][32][NT]  field g_i = 2 sum_{j != i} W_ij x_j + W_ii, so
+//   g     int32 [S][P][NT]   field g_i = 2 sum_{j != i} W_ij x_j + W_ii, so
 //                           Delta_i = phi(x_i) * g_i (Eq.(13)); pads INT32_MAX
 //   X,B,T uint8 [S][n_pad/8] bit vectors as little-endian bytes
 struct SearchState {
@@ -43,7 +54,7 @@ struct SearchState {
 struct RoundArgs {
     const int16_t *Wz;
     const int32_t *rowmax;
-    int32_t n, n_pad, nt;
+    int32_t n, n_pad, nt, bpt;
     int32_t *g;
     uint8_t *X;
     const uint8_t *T;
@@ -67,6 +78,6 @@ int launch_round(const RoundArgs &a, cudaStream_t st);
 // Delta int32 [count][n] (plain layout) or nothing.
 int launch_batch_init(const Instance &I, const uint8_t *X, int32_t count, int64_t *E, int32_t *delta,
                       cudaStream_t st);
-size_t round_smem_bytes(int32_t nt);
+size_t round_smem_bytes(int32_t nt, int32_t bpt);
 
 }  // namespace absb

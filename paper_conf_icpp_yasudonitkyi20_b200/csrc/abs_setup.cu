@@ -65,20 +65,20 @@ __global__ void rowmax_kernel(const int16_t *__restrict__ Wz, int n_pad, int32_t
 }
 
 // Device Step 1: C = 0, E = 0, Delta_i = W_ii (g_i = W_ii).
-__global__ void zero_start_kernel(int n, int nt, const int32_t *__restrict__ diag, int32_t *g, uint8_t *X,
+__global__ void zero_start_kernel(int n, int nt, int bpt, const int32_t *__restrict__ diag, int32_t *g, uint8_t *X,
                                   uint8_t *B, int64_t *E, int64_t *EB, int32_t *a, uint64_t *hash, int64_t *flips,
                                   int64_t *sflips, int s0)
 {
     const int sid = s0 + blockIdx.x;
     const int t = threadIdx.x;
-    int32_t *gs = g + (size_t)sid * 32 * nt;
-    for (int s = 0; s < 32; ++s) {
+    int32_t *gs = g + (size_t)sid * bpt * nt;
+    for (int s = 0; s < bpt; ++s) {
         const int i = slot_index(t, nt, s);
         gs[(size_t)s * nt + t] = (i < n) ? diag[i] : INT_MAX;  // pads are never candidates nor minima
     }
-    for (int j = 0; j < 4; ++j) {
-        X[(size_t)sid * 4 * nt + t + nt * j] = 0;
-        B[(size_t)sid * 4 * nt + t + nt * j] = 0;
+    for (int j = 0; j < bpt / 8; ++j) {
+        X[(size_t)sid * (bpt / 8) * nt + t + nt * j] = 0;
+        B[(size_t)sid * (bpt / 8) * nt + t + nt * j] = 0;
     }
     if (t == 0) {
         E[sid] = 0;
@@ -176,7 +176,7 @@ int launch_rowmax(const Instance &I, cudaStream_t st)
 int launch_zero_start(const Instance &I, SearchState &S, int32_t s0, int32_t s1, cudaStream_t st)
 {
     if (s1 <= s0) return 0;
-    zero_start_kernel<<<s1 - s0, I.nt, 0, st>>>(I.n, I.nt, I.diag, S.g, S.X, S.B, S.E, S.EB, S.a, S.hash, S.flips,
+    zero_start_kernel<<<s1 - s0, I.nt, 0, st>>>(I.n, I.nt, I.bpt, I.diag, S.g, S.X, S.B, S.E, S.EB, S.a, S.hash, S.flips,
                                                  S.sflips, s0);
     return (int)cudaGetLastError();
 }
