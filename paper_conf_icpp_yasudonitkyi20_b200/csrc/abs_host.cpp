@@ -311,6 +311,11 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
         const int rc2 = launch_rowmax(I, c->st);
         c->launches++;
         if (rc2) return bail(fail(ABS_ECUDA, std::string("rowmax: ") + cudaGetErrorString((cudaError_t)rc2)));
+        std::vector<int32_t> rm((size_t)I.n_pad);
+        CTX_CU(cudaMemcpyAsync(rm.data(), I.rowmax, sizeof(int32_t) * rm.size(), cudaMemcpyDeviceToHost, c->st));
+        CTX_CU(cudaStreamSynchronize(c->st));
+        I.wmax = 0;
+        for (int32_t v : rm) I.wmax = std::max(I.wmax, v);
     }
 
     // ---- per-search state
@@ -368,7 +373,7 @@ static int lockstep_step(abs_ctx *c)
     c->h2d += (int64_t)S * bpv;
     RoundArgs a{};
     a.Wz = c->I.Wz;
-    a.rowmax = c->I.rowmax;
+    a.wmax = c->I.wmax;
     a.n = c->I.n;
     a.n_pad = c->I.n_pad;
     a.nt = c->I.nt;

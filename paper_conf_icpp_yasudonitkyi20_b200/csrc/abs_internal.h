@@ -34,7 +34,8 @@ struct Instance {
     int32_t n = 0, n_pad = 0, nt = 0, bpt = 32;
     int16_t *Wz = nullptr;
     int32_t *diag = nullptr;
-    int32_t *rowmax = nullptr;  // [n_pad] max_i |W_ik| (i != k): bound on one flip's change of any Delta
+    int32_t *rowmax = nullptr;  // [n_pad] max_i |W_ik| (i != k)
+    int32_t wmax = 32768;       // max_{i != k} |W_ik|: one flip moves any Delta_i by at most 2*wmax
 };
 
 // Per-search state, structure of arrays (index = local search id).
@@ -53,7 +54,7 @@ struct SearchState {
 
 struct RoundArgs {
     const int16_t *Wz;
-    const int32_t *rowmax;
+    int32_t wmax;
     int32_t n, n_pad, nt, bpt;
     int32_t *g;
     uint8_t *X;

@@ -61,9 +61,9 @@ struct Red {
 
 // Shared-memory bookkeeping of a CTA (fixed size, at offset 0).
 struct RoundSmem {
-    uint64_t bar[2][8];   // [row buffer][chunk]
+    uint64_t bar[2][2];   // [row buffer][half row]
     Red red[2][32];
-    int sel[2][4];        // window warp -> all: next (k, Delta_k, x_k, exact_next), by flip parity
+    int4 sel[2];          // window warp -> all: next (k, Delta_k, x_k, exact_next), by flip parity
     int thr[2];           // improvement threshold E_B - E(X') clamped to int32, by flip parity
     long long E, EB, LB;  // E(X), E_B, lower bound on min_i Delta_i(X): thread 0 only
     unsigned long long hash;
@@ -215,7 +215,7 @@ struct Round {
         cmin = INT_MAX;
 #pragma unroll
         for (int j = 0; j < G; ++j) {
-            mbar_wait(&bars[j], par);
+            if (j % (G / 2) == 0) mbar_wait(&bars[j / (G / 2)], par);
             const uint4 w4 = row4[t + nt * j];
             const uint32_t wv[4] = {w4.x, w4.y, w4.z, w4.w};
 #pragma unroll
@@ -240,12 +240,12 @@ struct Round {
     static __device__ __forceinline__ void issue_row(const RoundArgs &A, int k, unsigned char *buf, uint64_t *bars,
                                                      int nt)
     {
-        const uint32_t chunk = 16u * (uint32_t)nt;
+        const uint32_t half = 8u * G * (uint32_t)nt;  // bytes of G/2 byte-groups = n_pad bytes
         const char *src = reinterpret_cast<const char *>(A.Wz) + (size_t)k * (size_t)A.n_pad * 2;
 #pragma unroll
-        for (int j = 0; j < G; ++j) {
-            mbar_arrive_expect_tx(&bars[j], chunk);
-            bulk_g2s(buf + (size_t)chunk * j, src + (size_t)chunk * j, chunk, &bars[j]);
+        for (int h = 0; h < 2; ++h) {
+            mbar_arrive_expect_tx(&bars[h], half);
+            bulk_g2s(buf + (size_t)half * h, src + (size_t)half * h, half, &bars[h]);
         }
     }
 
@@ -258,6 +258,14 @@ struct Round {
         const int b0 = a2 >> 3;
         const int b1 = (min(end, n) - 1) >> 3;
         const int b2 = end > n ? ((end - n - 1) >> 3) : -1;
+        if (kNT && (kNT & (kNT - 1)) == 0 && kNT > kWinMax / 8) {
+            // window spans < kNT bytes: thread t holds at most one byte of [b0, b1]
+            // (beta = b0 + ((t - b0) mod kNT)) and, if wrapped, byte t of [0, b2]
+            const int dlt = (t - b0) & (kNT - 1);
+            const int jw = dlt <= b1 - b0 ? (b0 + dlt) / kNT : -1;
+            const int jz = t <= b2 ? 0 : -1;
+            if (jw < 0 && jz < 0) return;
+        }
 #pragma unroll
         for (int j = 0; j < G; ++j) {
             const int beta = t + nt * j;
@@ -298,7 +306,7 @@ struct Round {
 #pragma unroll
             for (int b = 0; b < 2; ++b)
 #pragma unroll
-                for (int j = 0; j < G; ++j) mbar_init(&sm->bar[b][j], 1);
+                for (int h = 0; h < 2; ++h) mbar_init(&sm->bar[b][h], 1);
             fence_mbar_init();
             sm->hash = A.hash[sid];
             sm->nflip = 0;
@@ -353,11 +361,7 @@ struct Round {
             dk = r.c;
         }
         bool exact = true;  // compute the n neighbour deltas of this flip exactly
-        int rk = 0;         // thread 0: rowmax of the row being flipped
-        if (t == 0) {
-            rk = __ldg(A.rowmax + k);
-            issue_row(A, k, rowbuf, sm->bar[0], nt);
-        }
+        if (t == 0) issue_row(A, k, rowbuf, sm->bar[0], nt);
 
         for (int f = 0;; ++f) {
             const int b = f & 1;
@@ -365,19 +369,16 @@ struct Round {
             unsigned char *row = rowbuf + rowb * b;
 
             // ---- window-first selection of the next flip (warp 0), prefetch its row
-            int rk_next = 0;
             if (pre && !straight && left > 1 && warp == 0) {
                 int a1 = a + l;
                 if (a1 >= n) a1 -= n;
                 {
-                    // wait for the chunks of row k_f that hold the window's bits
+                    // wait for the half rows of row k_f that hold the window's bits
                     const int end = a1 + l - 1;
-                    const int c1 = group_of(min(end, n - 1), nt);
-                    for (int cc = group_of(a1, nt); cc <= c1; ++cc) mbar_wait(&sm->bar[b][cc], par);
-                    if (end >= n) {
-                        const int c2 = group_of(end - n, nt);
-                        for (int cc = 0; cc <= c2; ++cc) mbar_wait(&sm->bar[b][cc], par);
-                    }
+                    const int h0 = group_of(a1, nt) / (G / 2);
+                    const int h1 = (end >= n) ? 1 : group_of(end, nt) / (G / 2);
+                    if (end >= n || h0 == 0) mbar_wait(&sm->bar[b][0], par);
+                    if (h1 == 1) mbar_wait(&sm->bar[b][1], par);
                 }
                 const int *wd = win->d[b];
                 const uint8_t *wx = win->x[b];
@@ -426,10 +427,7 @@ struct Round {
                 const int mi = __reduce_min_sync(kFull, bv == mv ? 2 * bi + bx : INT_MAX);
                 if (lane == 0) {
                     issue_row(A, mi >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
-                    sm->sel[b][0] = mi >> 1;
-                    sm->sel[b][1] = mv;
-                    sm->sel[b][2] = mi & 1;
-                    rk_next = __ldg(A.rowmax + (mi >> 1));  // consumed after the row update
+                    sm->sel[b] = make_int4(mi >> 1, mv, mi & 1, 1);
                 }
             }
 
@@ -470,7 +468,7 @@ struct Round {
                 sm->nflip += 1;
                 if (straight) sm->nstraight += 1;
                 const long long E1 = sm->E + dk;
-                const long long LB1 = min(sm->LB - 2 * (long long)rk, -(long long)dk);
+                const long long LB1 = min(sm->LB - 2 * (long long)A.wmax, -(long long)dk);
                 const long long EB = sm->EB;
                 sm->E = E1;
                 sm->LB = LB1;
@@ -480,9 +478,9 @@ struct Round {
                 if (pre && !straight && left > 1) {
                     // E_B may still drop in this flip: the current (larger) E_B only makes
                     // the test more conservative
-                    const int dk1 = sm->sel[b][1];
-                    const long long LB2 = min(LB1 - 2 * (long long)rk_next, -(long long)dk1);
-                    sm->sel[b][3] = (E1 + dk1 + min(LB2, 0LL) < EB) ? 1 : 0;
+                    const int dk1 = sm->sel[b].y;
+                    const long long LB2 = min(LB1 - 2 * (long long)A.wmax, -(long long)dk1);
+                    sm->sel[b].w = (E1 + dk1 + min(LB2, 0LL) < EB) ? 1 : 0;
                 }
             }
 
@@ -526,11 +524,11 @@ struct Round {
             if (!straight) {
                 if (--left <= 0) break;
                 if (pre) {
-                    k = sm->sel[b][0];
-                    dk = sm->sel[b][1];
-                    xk = sm->sel[b][2];
-                    exact = sm->sel[b][3] != 0;
-                    rk = rk_next;
+                    const int4 sv = sm->sel[b];
+                    k = sv.x;
+                    dk = sv.y;
+                    xk = sv.z;
+                    exact = sv.w != 0;
                     continue;  // row already in flight
                 }
                 k = r1.i >> 1;
@@ -553,10 +551,7 @@ struct Round {
                 dk = r.c;
                 exact = true;
             }
-            if (t == 0) {
-                rk = __ldg(A.rowmax + k);
-                issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
-            }
+            if (t == 0) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
         }
 
         // ---- Step 5: store (B, E_B) and the state C' for the next round
