@@ -267,8 +267,18 @@ def run_abs(args):
     hbm = float(peaks.get("hbm_gbs", 6650.0))
     peak_src = "measured" if "hbm_gbs" in peaks else "fallback"
     achieved = flips * 2.0 * n / kern_s / 1e9 if kern_s > 0 else None
+    # traffic: DRAM bytes per flip of the round kernel from the committed ncu
+    # --set full capture (profiles/round_kernel_ncu.json), times this run's flips
+    # per launch; only for the workload it was captured on.
+    traffic = None
+    try:
+        prof = json.load(open(os.path.join(ROOT, "profiles", "round_kernel_ncu.json")))
+        if args.workload == "random32k" and launches > 0:
+            traffic = prof["dram_bytes_per_flip"] * flips / launches / 1e9
+    except Exception:
+        pass
     roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-            "frac": (achieved / hbm) if achieved else None, "traffic": None,
+            "frac": (achieved / hbm) if achieved else None, "traffic": traffic, "traffic_unit": "GB per launch",
             "peak_source": peak_src, "kernel": "round_kernel",
             "algorithmic_bytes_per_launch": flips * 2.0 * n / max(1, launches),
             "avg_launch_ms": 1e3 * kern_s / max(1, launches),
