@@ -217,8 +217,10 @@ def run_abs(args):
     L = args.local_flips or n
     Wp = torch.from_numpy(W).pin_memory()
     Wd = Wp.to(f"cuda:{local}", non_blocking=False)
-    common = dict(searches=S, local_flips=L, pool_size=64, seed=1, device=local)
-    solver = pkg.Solver(Wd, search_offset=rank * S, external_merge=(world > 1), **common)
+    mode = pkg.MODE_ASYNC if args.mode == "async" else pkg.MODE_LOCKSTEP
+    common = dict(searches=S, local_flips=L, pool_size=64, seed=1, device=local, mode=mode)
+    solver = pkg.Solver(Wd, search_offset=rank * S, external_merge=(world > 1 and mode == pkg.MODE_LOCKSTEP),
+                        **common)
     del Wd
 
     def step(s):
@@ -227,8 +229,18 @@ def run_abs(args):
         else:
             s.search(1)
 
-    for _ in range(args.warmup):
-        step(solver)
+    def run_steps(s, k):
+        if mode == pkg.MODE_ASYNC:
+            # one persistent launch for all k rounds of every search (the
+            # blocks run asynchronously); ranks then all-gather their elites
+            s.search(k)
+            if world > 1:
+                pdist.exchange_elites(s, 64)
+        else:
+            for _ in range(k):
+                step(s)
+
+    run_steps(solver, args.warmup)
     barrier()
     torch.cuda.synchronize()
     st0 = solver.stats()
@@ -237,8 +249,7 @@ def run_abs(args):
         barrier()
         torch.cuda.synchronize()
         ev0.record()
-        for _ in range(args.steps):
-            step(solver)
+        run_steps(solver, args.steps)
         ev1.record()
         torch.cuda.synchronize()
         barrier()
@@ -294,9 +305,9 @@ def run_abs(args):
         torch.cuda.synchronize()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        s2 = pkg.Solver(Wp.numpy(), search_offset=rank * S, external_merge=(world > 1), **common)
-        for _ in range(args.steps):
-            step(s2)
+        s2 = pkg.Solver(Wp.numpy(), search_offset=rank * S,
+                        external_merge=(world > 1 and mode == pkg.MODE_LOCKSTEP), **common)
+        run_steps(s2, args.steps)
         Xb, Eb = s2.best() if world == 1 else (None, None)
         e1.record()
         torch.cuda.synchronize()
@@ -331,7 +342,7 @@ def run_abs(args):
             "data": "synthetic (Philox random int16 QUBO, P:L468)" if args.workload.startswith("random")
             else "synthetic",
             "config": {"workload": args.workload, "desc": WORKLOADS[args.workload], "n": n,
-                       "searches_per_gpu": S, "local_flips": L, "pool": 64, "mode": "lockstep",
+                       "searches_per_gpu": S, "local_flips": L, "pool": 64, "mode": args.mode,
                        "parallelism": "dp%d (replicated W, independent searches)" % world,
                        "l2": "inputs larger than L2 (W = %d MiB)" % (2 * n * n >> 20)
                        if 2 * n * n > 126 * 2 ** 20 else "W fits in L2 (resident by design)"},
@@ -357,6 +368,7 @@ def main():
     ap.add_argument("--impl", default="abs", choices=["abs", "reference"])
     ap.add_argument("--workload", default="random32k", choices=sorted(WORKLOADS))
     ap.add_argument("--searches", type=int, default=0)
+    ap.add_argument("--mode", default="lockstep", choices=["lockstep", "async"])
     ap.add_argument("--local-flips", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -84,7 +84,10 @@ typedef struct abs_config {
                              * results of all ranks with abs_pool_insert (in
                              * global search-id order) before the next step */
     int32_t device;         /* CUDA device ordinal; -1 -> current device */
-    int32_t reserved[8];    /* must be 0 */
+    int32_t trace;          /* async only: 1 = record, per round, the target the
+                             * search used and its (B, E_B) (abs_trace_*), so a
+                             * run can be replayed exactly; costs host memory */
+    int32_t reserved[7];    /* must be 0 */
 } abs_config;
 
 typedef struct abs_stats {
@@ -171,6 +174,15 @@ ABS_API int abs_round_results(const abs_ctx *c, uint32_t *B_out, int64_t *EB_out
 
 /* Lockstep: the targets T the searches used in the last step. */
 ABS_API int abs_round_targets(const abs_ctx *c, uint32_t *T_out);
+
+/* Async trace (cfg.trace = 1): number of recorded rounds. */
+ABS_API int abs_trace_count(const abs_ctx *c, int64_t *count);
+
+/* Async trace entry i (arrival order): local search index, round number,
+ * the target T the round used (words(n)), and its (B, E_B).  Any output may
+ * be NULL. */
+ABS_API int abs_trace_get(const abs_ctx *c, int64_t i, int32_t *s_out, int32_t *round_out, uint32_t *T_out,
+                          uint32_t *B_out, int64_t *EB_out);
 
 /* Per-search state (debug / parity): current solution C (words(n)), Delta
  * (n int32), E, window offset a, window length l, FNV-1a-64 hash of the flip

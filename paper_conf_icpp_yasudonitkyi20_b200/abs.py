@@ -44,7 +44,8 @@ class abs_config(C.Structure):
         ("mode", C.c_int32),
         ("external_merge", C.c_int32),
         ("device", C.c_int32),
-        ("reserved", C.c_int32 * 8),
+        ("trace", C.c_int32),
+        ("reserved", C.c_int32 * 7),
     ]
 
 
@@ -72,7 +73,7 @@ class abs_stats(C.Structure):
 EXPORTS = [
     "abs_config_init", "abs_create", "abs_create_dev", "abs_seed_pool", "abs_search", "abs_best",
     "abs_stats_get", "abs_pool_get", "abs_pool_insert", "abs_energy", "abs_round_results",
-    "abs_round_targets", "abs_search_state", "abs_destroy", "abs_strerror", "abs_last_error", "abs_version",
+    "abs_round_targets", "abs_trace_count", "abs_trace_get", "abs_search_state", "abs_destroy", "abs_strerror", "abs_last_error", "abs_version",
 ]
 
 _lib = None
@@ -112,6 +113,8 @@ def load(build_if_missing: bool = True):
     L.abs_energy.argtypes = [vp, vp, C.c_int32, vp, vp]
     L.abs_round_results.argtypes = [vp, vp, vp]
     L.abs_round_targets.argtypes = [vp, vp]
+    L.abs_trace_count.argtypes = [vp, P(C.c_int64)]
+    L.abs_trace_get.argtypes = [vp, C.c_int64, P(C.c_int32), P(C.c_int32), vp, vp, P(C.c_int64)]
     L.abs_search_state.argtypes = [vp, C.c_int32, vp, vp, P(C.c_int64), P(C.c_int32), P(C.c_int32),
                                    P(C.c_uint64), P(C.c_int64)]
     L.abs_destroy.argtypes = [vp]
@@ -153,7 +156,7 @@ def words(n: int) -> int:
 def make_config(n: int, searches: int = 148, search_offset: int = 0, local_flips: int | None = None,
                 pool_size: int = 64, ladder=None, seed: int = 1, p_cross: int = -1, p_mut: int = -1,
                 mut_max: int = 0, mode: int = MODE_LOCKSTEP, external_merge: bool = False,
-                device: int = -1) -> abs_config:
+                device: int = -1, trace: bool = False) -> abs_config:
     cfg = abs_config()
     load().abs_config_init(C.byref(cfg))
     cfg.searches = int(searches)
@@ -173,6 +176,7 @@ def make_config(n: int, searches: int = 148, search_offset: int = 0, local_flips
     cfg.mode = int(mode)
     cfg.external_merge = 1 if external_merge else 0
     cfg.device = int(device)
+    cfg.trace = 1 if trace else 0
     return cfg
 
 
@@ -279,6 +283,20 @@ class Solver:
         T = np.zeros((self.searches, self.words), np.uint32)
         _check(load().abs_round_targets(self._c, _ptr(T)), "abs_round_targets")
         return T
+
+    def trace(self):
+        """Async trace: list of (search, round, T, B, E_B) in arrival order."""
+        cnt = C.c_int64()
+        _check(load().abs_trace_count(self._c, C.byref(cnt)), "abs_trace_count")
+        out = []
+        for i in range(cnt.value):
+            s, r, EB = C.c_int32(), C.c_int32(), C.c_int64()
+            T = np.zeros(self.words, np.uint32)
+            B = np.zeros(self.words, np.uint32)
+            _check(load().abs_trace_get(self._c, i, C.byref(s), C.byref(r), _ptr(T), _ptr(B), C.byref(EB)),
+                   "abs_trace_get")
+            out.append((s.value, r.value, T, B, int(EB.value)))
+        return out
 
     def search_state(self, s: int) -> dict:
         X = np.zeros(self.words, np.uint32)

@@ -131,6 +131,12 @@ static void ga_target(const Pool &P, const GaParams &ga, int64_t r, int64_t sid,
 
 using namespace absb;
 
+struct TraceEntry {
+    int32_t s, round;
+    std::vector<uint32_t> T, B;
+    int64_t EB;
+};
+
 struct abs_ctx {
     abs_config cfg{};
     int device = 0;
@@ -152,6 +158,19 @@ struct abs_ctx {
     int64_t rounds_done = 0, pool_inserted = 0, steps = 0;
     int64_t h2d = 0, d2h = 0, launches = 0, round_launches = 0;
     double step_seconds = 0.0;
+    // ---- asynchronous mode (the paper's Fig. 5): mapped pinned exchange buffers
+    bool async_ready = false;
+    uint8_t *Tmap = nullptr;                     // [S][2][bpv] host view
+    uint32_t *tseq = nullptr, *rtver = nullptr, *rseq = nullptr, *rack = nullptr;
+    uint8_t *Rb = nullptr;                       // [S][2][bpv]
+    int64_t *Reb = nullptr;                      // [S][2]
+    unsigned int *rcount = nullptr;
+    unsigned long long *queue_d = nullptr;
+    int *done_d = nullptr;
+    std::vector<uint32_t> tver, consumed;        // host-side per-search versions / consumed rounds
+    std::vector<std::vector<std::vector<uint32_t>>> hist;  // trace: targets by version
+    std::vector<TraceEntry> trace;
+    int async_grid = 0;
 };
 
 static void free_ctx(abs_ctx *c)
@@ -176,6 +195,16 @@ static void free_ctx(abs_ctx *c)
     if (c->T_h) cudaFreeHost(c->T_h);
     if (c->B_h) cudaFreeHost(c->B_h);
     if (c->EB_h) cudaFreeHost(c->EB_h);
+    if (c->Tmap) cudaFreeHost(c->Tmap);
+    if (c->tseq) cudaFreeHost(c->tseq);
+    if (c->rtver) cudaFreeHost(c->rtver);
+    if (c->rseq) cudaFreeHost(c->rseq);
+    if (c->rack) cudaFreeHost(c->rack);
+    if (c->Rb) cudaFreeHost(c->Rb);
+    if (c->Reb) cudaFreeHost(c->Reb);
+    if (c->rcount) cudaFreeHost(c->rcount);
+    cudaFree(c->queue_d);
+    cudaFree(c->done_d);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
     if (c->evs0) cudaEventDestroy(c->evs0);
@@ -417,6 +446,173 @@ static int lockstep_step(abs_ctx *c)
     return ABS_OK;
 }
 
+// ------------------------------------------------------------------ asynchronous mode
+template <typename T>
+static T vload(const T *p)
+{
+    return *reinterpret_cast<const volatile T *>(p);
+}
+template <typename T>
+static void vstore(T *p, T v)
+{
+    *reinterpret_cast<volatile T *>(p) = v;
+}
+
+static int async_setup(abs_ctx *c)
+{
+    const int S = c->S.S, bpv = c->bytes_per_vec;
+    const unsigned fl = cudaHostAllocMapped | cudaHostAllocPortable;
+    ABS_CU(cudaHostAlloc(&c->Tmap, (size_t)S * 2 * bpv, fl));
+    ABS_CU(cudaHostAlloc(&c->Rb, (size_t)S * 2 * bpv, fl));
+    ABS_CU(cudaHostAlloc(&c->Reb, (size_t)S * 2 * sizeof(int64_t), fl));
+    ABS_CU(cudaHostAlloc(&c->tseq, (size_t)S * sizeof(uint32_t), fl));
+    ABS_CU(cudaHostAlloc(&c->rtver, (size_t)S * 2 * sizeof(uint32_t), fl));
+    ABS_CU(cudaHostAlloc(&c->rseq, (size_t)S * sizeof(uint32_t), fl));
+    ABS_CU(cudaHostAlloc(&c->rack, (size_t)S * sizeof(uint32_t), fl));
+    ABS_CU(cudaHostAlloc(&c->rcount, sizeof(unsigned int), fl));
+    std::memset(c->Tmap, 0, (size_t)S * 2 * bpv);
+    std::memset(c->Rb, 0, (size_t)S * 2 * bpv);
+    std::memset(c->tseq, 0, (size_t)S * sizeof(uint32_t));
+    std::memset(c->rseq, 0, (size_t)S * sizeof(uint32_t));
+    std::memset(c->rack, 0, (size_t)S * sizeof(uint32_t));
+    *c->rcount = 0;
+    ABS_CU(cudaMalloc(&c->queue_d, sizeof(unsigned long long)));
+    ABS_CU(cudaMalloc(&c->done_d, (size_t)S * sizeof(int)));
+    ABS_CU(cudaMemset(c->done_d, 0, (size_t)S * sizeof(int)));
+    c->tver.assign(S, 0);
+    c->consumed.assign(S, 0);
+    if (c->cfg.trace) c->hist.assign(S, {});
+    // round-0 targets from the initial pool (host Step 1 + Step 4)
+    std::vector<uint32_t> T(c->pool.words);
+    for (int s = 0; s < S; ++s) {
+        ga_target(c->pool, c->ga, c->round, (int64_t)c->cfg.search_offset + s, T.data());
+        std::memcpy(c->Tmap + ((size_t)s * 2 + 1) * bpv, T.data(), sizeof(uint32_t) * T.size());
+        c->tver[s] = 1;
+        if (c->cfg.trace) c->hist[s].assign(2, {}), c->hist[s][1] = T;
+    }
+    std::atomic_thread_fence(std::memory_order_release);
+    for (int s = 0; s < S; ++s) vstore(c->tseq + s, 1u);
+    c->async_ready = true;
+    return ABS_OK;
+}
+
+// Host Steps 2-4 for every result published so far: insert it
+// into the pool, acknowledge the slot, generate one new target for the search.
+static void async_consume(abs_ctx *c)
+{
+    const int S = c->S.S, bpv = c->bytes_per_vec, words = c->pool.words;
+    std::vector<uint32_t> B(words), T(words);
+    for (int s = 0; s < S; ++s) {
+        const uint32_t rs = vload(c->rseq + s);
+        if (rs <= c->consumed[s]) continue;
+        std::atomic_thread_fence(std::memory_order_acquire);
+        while (c->consumed[s] < rs) {
+            const uint32_t r = c->consumed[s];
+            const size_t slot = (size_t)s * 2 + (r & 1);
+            std::memcpy(B.data(), c->Rb + slot * bpv, sizeof(uint32_t) * words);
+            const int64_t EB = vload(c->Reb + slot);
+            const uint32_t v = vload(c->rtver + slot);
+            c->pool_inserted += c->pool.insert(B.data(), EB) ? 1 : 0;  // Step 3
+            if (c->cfg.trace) c->trace.push_back(TraceEntry{s, (int32_t)r, c->hist[s][v], B, EB});
+            c->consumed[s] = r + 1;
+            std::atomic_thread_fence(std::memory_order_release);
+            vstore(c->rack + s, r + 1);
+            // Step 4: "as many new target solutions as newly arrived solutions"
+            ga_target(c->pool, c->ga, (int64_t)r + 1, (int64_t)c->cfg.search_offset + s, T.data());
+            const uint32_t nv = c->tver[s] + 1;
+            std::memcpy(c->Tmap + ((size_t)s * 2 + (nv & 1)) * bpv, T.data(), sizeof(uint32_t) * words);
+            if (c->cfg.trace) c->hist[s].push_back(T);
+            std::atomic_thread_fence(std::memory_order_release);
+            vstore(c->tseq + s, nv);
+            c->tver[s] = nv;
+        }
+    }
+}
+
+static int async_run(abs_ctx *c, int64_t steps)
+{
+    if (!c->async_ready) {
+        const int rc = async_setup(c);
+        if (rc) return rc;
+    }
+    const int S = c->S.S;
+    if ((int64_t)c->round + steps > INT32_MAX) return fail(ABS_EINVAL, "too many rounds");
+    ABS_CU(cudaMemsetAsync(c->queue_d, 0, sizeof(unsigned long long), c->st));
+    AsyncArgs q{};
+    auto dev = [](auto *h) {
+        void *d = nullptr;
+        cudaHostGetDevicePointer(&d, (void *)h, 0);
+        return d;
+    };
+    q.queue = c->queue_d;
+    q.total = (long long)S * steps;
+    q.base = (int)c->round;
+    q.done = c->done_d;
+    q.Tmap = (const uint8_t *)dev(c->Tmap);
+    q.tseq = (const uint32_t *)dev(c->tseq);
+    q.Rb = (uint8_t *)dev(c->Rb);
+    q.Reb = (int64_t *)dev(c->Reb);
+    q.rtver = (uint32_t *)dev(c->rtver);
+    q.rseq = (uint32_t *)dev(c->rseq);
+    q.rack = (const uint32_t *)dev(c->rack);
+    q.rcount = (unsigned int *)dev(c->rcount);
+    RoundArgs a{};
+    a.Wz = c->I.Wz;
+    a.wmax = c->I.wmax;
+    a.n = c->I.n;
+    a.n_pad = c->I.n_pad;
+    a.nt = c->I.nt;
+    a.bpt = c->I.bpt;
+    a.g = c->S.g;
+    a.X = c->S.X;
+    a.T = nullptr;
+    a.B = c->S.B;
+    a.E = c->S.E;
+    a.EB = c->S.EB;
+    a.a = c->S.a;
+    a.l = c->S.l;
+    a.hash = c->S.hash;
+    a.flips = c->S.flips;
+    a.sflips = c->S.sflips;
+    a.L = c->L;
+    a.S = S;
+
+    // the host GA thread, concurrent with the persistent kernel
+    std::atomic<bool> stop{false};
+    std::thread ga([c, &stop]() {
+        unsigned int seen = 0;
+        for (;;) {
+            const bool last = stop.load(std::memory_order_acquire);
+            const unsigned int cnt = vload(c->rcount);  // Step 2: poll the global counter
+            if (cnt != seen || last) {
+                seen = cnt;
+                async_consume(c);
+                if (last) break;
+            } else {
+                std::this_thread::sleep_for(std::chrono::microseconds(20));
+            }
+        }
+    });
+    ABS_CU(cudaEventRecord(c->ev0, c->st));
+    const int rc = launch_round(a, c->st, &q, &c->async_grid);
+    c->launches++;
+    c->round_launches++;
+    cudaError_t e1 = cudaEventRecord(c->ev1, c->st);
+    cudaError_t e2 = cudaStreamSynchronize(c->st);
+    stop.store(true, std::memory_order_release);
+    ga.join();  // drains every published result
+    if (rc) return fail(ABS_ECUDA, std::string("round_kernel_async: ") + cudaGetErrorString((cudaError_t)rc));
+    ABS_CU(e1);
+    ABS_CU(e2);
+    float ms = 0.f;
+    ABS_CU(cudaEventElapsedTime(&ms, c->ev0, c->ev1));
+    c->search_seconds += ms * 1e-3;
+    c->rounds_done += (int64_t)S * steps;
+    c->round += steps;
+    c->steps += steps;
+    return ABS_OK;
+}
+
 extern "C" {
 
 void abs_config_init(abs_config *cfg)
@@ -521,11 +717,15 @@ int abs_search(abs_ctx *c, int64_t steps)
     if (c->S.S == 0 || steps == 0) return ABS_OK;
     try {
         ABS_CU(cudaSetDevice(c->device));
-        if (c->cfg.mode != ABS_MODE_LOCKSTEP) return fail(ABS_EINVAL, "async mode not available in this build");
         ABS_CU(cudaEventRecord(c->evs0, c->st));
-        for (int64_t s = 0; s < steps; ++s) {
-            const int rc = lockstep_step(c);
+        if (c->cfg.mode == ABS_MODE_ASYNC) {
+            const int rc = async_run(c, steps);
             if (rc) return rc;
+        } else {
+            for (int64_t s = 0; s < steps; ++s) {
+                const int rc = lockstep_step(c);
+                if (rc) return rc;
+            }
         }
         ABS_CU(cudaEventRecord(c->evs1, c->st));
         ABS_CU(cudaEventSynchronize(c->evs1));
@@ -608,7 +808,7 @@ int abs_pool_insert(abs_ctx *c, const uint32_t *X, const int64_t *E, int32_t cou
 int abs_round_results(const abs_ctx *c, uint32_t *B_out, int64_t *EB_out)
 {
     if (!c || !B_out || !EB_out) return fail(ABS_EINVAL, "bad arguments");
-    if (!c->have_results) return fail(ABS_ESTATE, "no round has run");
+    if (!c->have_results || c->cfg.mode != ABS_MODE_LOCKSTEP) return fail(ABS_ESTATE, "no lockstep round has run");
     const int words = c->pool.words;
     for (int s = 0; s < c->S.S; ++s) {
         std::memcpy(B_out + (size_t)s * words, c->B_h + (size_t)s * c->bytes_per_vec, sizeof(uint32_t) * words);
@@ -624,6 +824,26 @@ int abs_round_targets(const abs_ctx *c, uint32_t *T_out)
     const int words = c->pool.words;
     for (int s = 0; s < c->S.S; ++s)
         std::memcpy(T_out + (size_t)s * words, c->T_h + (size_t)s * c->bytes_per_vec, sizeof(uint32_t) * words);
+    return ABS_OK;
+}
+
+int abs_trace_count(const abs_ctx *c, int64_t *count)
+{
+    if (!c || !count) return fail(ABS_EINVAL, "bad arguments");
+    *count = (int64_t)c->trace.size();
+    return ABS_OK;
+}
+
+int abs_trace_get(const abs_ctx *c, int64_t i, int32_t *s_out, int32_t *round_out, uint32_t *T_out, uint32_t *B_out,
+                  int64_t *EB_out)
+{
+    if (!c || i < 0 || i >= (int64_t)c->trace.size()) return fail(ABS_EINVAL, "bad arguments");
+    const TraceEntry &e = c->trace[(size_t)i];
+    if (s_out) *s_out = e.s;
+    if (round_out) *round_out = e.round;
+    if (T_out) std::copy(e.T.begin(), e.T.end(), T_out);
+    if (B_out) std::copy(e.B.begin(), e.B.end(), B_out);
+    if (EB_out) *EB_out = e.EB;
     return ABS_OK;
 }
 

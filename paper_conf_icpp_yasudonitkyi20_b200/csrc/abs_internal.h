@@ -69,12 +69,31 @@ struct RoundArgs {
     int32_t S;
 };
 
+// Asynchronous mode (ABS_MODE_ASYNC): work queue and the host<->device
+// exchange buffers (mapped pinned host memory, device pointers).
+struct AsyncArgs {
+    unsigned long long *queue;  // device: next work item (search, round) = (q % S, base + q / S)
+    long long total;            // items of this launch = S * steps
+    int base;                   // rounds every search had completed before this launch
+    int *done;                  // device [S]: rounds completed per search
+    const uint8_t *Tmap;        // mapped [S][2][n_pad/8]: double-buffered targets
+    const uint32_t *tseq;       // mapped [S]: latest target version (slot = version & 1)
+    uint8_t *Rb;                // mapped [S][2][n_pad/8]: B of round r in slot r & 1
+    int64_t *Reb;               // mapped [S][2]: E_B
+    uint32_t *rtver;            // mapped [S][2]: target version the round used
+    uint32_t *rseq;             // mapped [S]: rounds published
+    const uint32_t *rack;       // mapped [S]: rounds consumed by the host
+    unsigned int *rcount;       // mapped: total results published (polled by the host GA)
+};
+
 // Launchers (return cudaError_t as int).
 int launch_prepare_w(const int16_t *W_in, int32_t n, int32_t n_pad, int16_t *Wz, int32_t *diag,
                      unsigned long long *asym_count, cudaStream_t st);
 int launch_rowmax(const Instance &I, cudaStream_t st);
 int launch_zero_start(const Instance &I, SearchState &S, int32_t s0, int32_t s1, cudaStream_t st);
-int launch_round(const RoundArgs &a, cudaStream_t st);
+// q == nullptr: lockstep round (one CTA per search); otherwise the persistent
+// asynchronous kernel (grid = min(S, resident CTAs), *grid_out).
+int launch_round(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q = nullptr, int *grid_out = nullptr);
 // Batched init: X bytes [count][n_pad/8] -> E [count], and either
 // Delta int32 [count][n] (plain layout) or nothing.
 int launch_batch_init(const Instance &I, const uint8_t *X, int32_t count, int64_t *E, int32_t *delta,

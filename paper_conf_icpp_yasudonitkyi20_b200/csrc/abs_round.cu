@@ -29,6 +29,7 @@
 // every Delta_i, i != k, by at most 2*max_i|W_ik|, and Delta_k becomes
 // -Delta_k), and a flip whose bound already rules out an improvement skips the
 // n readouts; the result (B, E_B) is identical by construction.
+#include <algorithm>
 #include <climits>
 #include <cstdint>
 
@@ -92,7 +93,7 @@ struct Round {
     static __device__ __forceinline__ int group_of(int i, int nt)
     {
         const int beta = i >> 3;
-        if (kNT) return beta / kNT;
+        if constexpr (kNT != 0) return beta / kNT;
         int j = 0;
 #pragma unroll
         for (int m = 1; m < G; ++m) j += (beta >= m * nt);
@@ -258,7 +259,7 @@ struct Round {
         const int b0 = a2 >> 3;
         const int b1 = (min(end, n) - 1) >> 3;
         const int b2 = end > n ? ((end - n - 1) >> 3) : -1;
-        if (kNT && (kNT & (kNT - 1)) == 0 && kNT > kWinMax / 8) {
+        if constexpr (kNT != 0 && (kNT & (kNT - 1)) == 0 && kNT > kWinMax / 8) {
             // window spans < kNT bytes: thread t holds at most one byte of [b0, b1]
             // (beta = b0 + ((t - b0) mod kNT)) and, if wrapped, byte t of [0, b2]
             const int dlt = (t - b0) & (kNT - 1);
@@ -285,14 +286,31 @@ struct Round {
         }
     }
 
+    static __device__ __forceinline__ void init_barriers(unsigned char *smem)
+    {
+        RoundSmem *sm = reinterpret_cast<RoundSmem *>(smem);
+        if (threadIdx.x == 0) {
+#pragma unroll
+            for (int b = 0; b < 2; ++b)
+#pragma unroll
+                for (int h = 0; h < 2; ++h) mbar_init(&sm->bar[b][h], 1);
+            fence_mbar_init();
+        }
+        // made visible by the first barrier of run()
+    }
+
     // ---------------------------------------------------------------- the round
-    static __device__ __forceinline__ void run(const RoundArgs &A, unsigned char *smem)
+    // One round of search `sid`: target bits from Ts, (B, E_B) to Bs_out / *EB_out.
+    // fbase counts the rows this CTA has consumed before (row buffer and mbarrier
+    // phase of flip f are those of use fbase + f); the barriers are initialised
+    // once per launch by init_barriers().
+    static __device__ __forceinline__ void run(const RoundArgs &A, unsigned char *smem, int sid, const uint8_t *Ts,
+                                               uint8_t *Bs_out, int64_t *EB_out, int &fbase)
     {
         const int nt = kNT ? kNT : (kMulti ? A.nt : 32);
         const int n = A.n;
         const int t = threadIdx.x;
         const int lane = t & 31, warp = t >> 5, nw = nt >> 5;
-        const int sid = blockIdx.x;
         const size_t rowb = (size_t)2 * kP * nt;  // bytes of one padded row (2 * n_pad)
 
         RoundSmem *sm = reinterpret_cast<RoundSmem *>(smem);
@@ -303,11 +321,6 @@ struct Round {
             smem + ((sizeof(RoundSmem) + (kMulti ? sizeof(WindowSmem) : 0) + 2 * sizeof(M) * nt + 127) & ~size_t(127));
 
         if (t == 0) {
-#pragma unroll
-            for (int b = 0; b < 2; ++b)
-#pragma unroll
-                for (int h = 0; h < 2; ++h) mbar_init(&sm->bar[b][h], 1);
-            fence_mbar_init();
             sm->hash = A.hash[sid];
             sm->nflip = 0;
             sm->nstraight = 0;
@@ -326,7 +339,6 @@ struct Round {
         M xm = 0;
         {
             const uint8_t *Xs = A.X + (size_t)sid * G * nt;
-            const uint8_t *Ts = A.T + (size_t)sid * G * nt;
             M tm = 0;
 #pragma unroll
             for (int j = 0; j < G; ++j) {
@@ -353,7 +365,7 @@ struct Round {
             if (pre && !straight) {
                 int a2 = a + l;
                 if (a2 >= n) a2 -= n;
-                publish_window(g, xm, a2, l, n, t, nt, win->d[0], win->x[0]);
+                publish_window(g, xm, a2, l, n, t, nt, win->d[fbase & 1], win->x[fbase & 1]);
             }
             const Red r = block_reduce(Red{INT_MAX, cv, ci2}, sm->red, rb, lane, warp, nw);
             k = r.i >> 1;
@@ -361,11 +373,12 @@ struct Round {
             dk = r.c;
         }
         bool exact = true;  // compute the n neighbour deltas of this flip exactly
-        if (t == 0) issue_row(A, k, rowbuf, sm->bar[0], nt);
+        if (t == 0) issue_row(A, k, rowbuf + rowb * (fbase & 1), sm->bar[fbase & 1], nt);
 
-        for (int f = 0;; ++f) {
-            const int b = f & 1;
-            const uint32_t par = (uint32_t)(f >> 1) & 1u;
+        int f = 0;
+        for (;; ++f) {
+            const int b = (fbase + f) & 1;
+            const uint32_t par = (uint32_t)((fbase + f) >> 1) & 1u;
             unsigned char *row = rowbuf + rowb * b;
 
             // ---- window-first selection of the next flip (warp 0), prefetch its row
@@ -554,6 +567,8 @@ struct Round {
             if (t == 0) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
         }
 
+        fbase += f + 1;  // rows consumed in this round (no row left in flight)
+
         // ---- Step 5: store (B, E_B) and the state C' for the next round
         sync();
         {
@@ -561,16 +576,16 @@ struct Round {
 #pragma unroll
             for (int s = 0; s < kP; ++s) gs[(size_t)s * nt + t] = g[s];
             uint8_t *Xs = A.X + (size_t)sid * G * nt;
-            uint8_t *Bs = A.B + (size_t)sid * G * nt;
             const M bm = sbm[t];
 #pragma unroll
             for (int j = 0; j < G; ++j) {
                 Xs[t + nt * j] = (uint8_t)(xm >> (8 * j));
-                Bs[t + nt * j] = (uint8_t)(bm >> (8 * j));
+                Bs_out[t + nt * j] = (uint8_t)(bm >> (8 * j));
             }
             if (t == 0) {
                 A.E[sid] = sm->E;
                 A.EB[sid] = sm->EB;
+                *EB_out = sm->EB;
                 A.a[sid] = a;
                 A.hash[sid] = sm->hash;
                 A.flips[sid] += sm->nflip;
@@ -584,15 +599,102 @@ template <int kP, int kMaxT, int kNT>
 __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? 32 : (kMaxT == 128 ? 6 : 1)) round_kernel(const RoundArgs A)
 {
     extern __shared__ __align__(128) unsigned char smem[];
-    Round<kP, kMaxT, kNT>::run(A, smem);
+    const int sid = blockIdx.x;
+    const size_t bpv = (size_t)A.n_pad / 8;
+    int fbase = 0;
+    Round<kP, kMaxT, kNT>::init_barriers(smem);
+    Round<kP, kMaxT, kNT>::run(A, smem, sid, A.T + sid * bpv, A.B + sid * bpv, A.EB + sid, fbase);
+}
+
+// ---------------------------------------------------------------- asynchronous mode
+__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t *p)
+{
+    uint32_t v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_sys(uint32_t *p, uint32_t v)
+{
+    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ int ld_acquire_gpu(const int *p)
+{
+    int v;
+    asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ void st_release_gpu(int *p, int v)
+{
+    asm volatile("st.release.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+
+// The paper's device loop (Steps 2-5 repeated) as a persistent
+// kernel: CTAs take (search, round) items from a queue, read the search's
+// latest target from mapped host memory (Step 2; a stale target is reused,
+// reading C11), run the round, and publish (B, E_B) to mapped host memory
+// with a system-scope release plus a global counter the host GA polls
+// (P:L408).  Host and device never synchronise directly.
+template <int kP, int kMaxT, int kNT>
+__global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? 32 : (kMaxT == 128 ? 6 : 1))
+    round_kernel_async(const RoundArgs A, const AsyncArgs Q)
+{
+    extern __shared__ __align__(128) unsigned char smem[];
+    __shared__ long long item;
+    __shared__ uint32_t tver;
+    const size_t bpv = (size_t)A.n_pad / 8;
+    constexpr bool multi = kMaxT > 32;
+    int fbase = 0;
+    Round<kP, kMaxT, kNT>::init_barriers(smem);
+    for (;;) {
+        if (threadIdx.x == 0) item = (long long)atomicAdd(Q.queue, 1ull);
+        if (multi) __syncthreads();
+        else __syncwarp();
+        const long long q = item;
+        if (q >= Q.total) break;
+        const int s = (int)(q % A.S);
+        const int r = Q.base + (int)(q / A.S);
+        if (threadIdx.x == 0) {
+            while (ld_acquire_gpu(Q.done + s) != r) __nanosleep(256);  // round r-1 of s finished
+            // the result slot of round r (double-buffered) must have been consumed by the host
+            while ((int)ld_acquire_sys(Q.rack + s) < r - 1) __nanosleep(1024);
+            tver = ld_acquire_sys(Q.tseq + s);  // latest published target version
+        }
+        if (multi) __syncthreads();
+        else __syncwarp();
+        const uint32_t v = tver;
+        Round<kP, kMaxT, kNT>::run(A, smem, s, Q.Tmap + ((size_t)s * 2 + (v & 1)) * bpv,
+                                   Q.Rb + ((size_t)s * 2 + (r & 1)) * bpv, Q.Reb + (size_t)s * 2 + (r & 1), fbase);
+        __threadfence_system();
+        if (multi) __syncthreads();
+        else __syncwarp();
+        if (threadIdx.x == 0) {
+            Q.rtver[(size_t)s * 2 + (r & 1)] = v;
+            __threadfence_system();
+            st_release_sys(Q.rseq + s, (uint32_t)(r + 1));
+            atomicAdd_system(Q.rcount, 1u);
+            st_release_gpu(Q.done + s, r + 1);
+        }
+    }
 }
 
 template <int kP, int kMaxT, int kNT>
-int launch_variant(const RoundArgs &a, cudaStream_t st, size_t smem)
+int launch_variant(const RoundArgs &a, cudaStream_t st, size_t smem, const AsyncArgs *q, int *grid_out)
 {
-    auto k = round_kernel<kP, kMaxT, kNT>;
+    if (!q) {
+        auto k = round_kernel<kP, kMaxT, kNT>;
+        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        k<<<a.S, a.nt, smem, st>>>(a);
+        return (int)cudaGetLastError();
+    }
+    auto k = round_kernel_async<kP, kMaxT, kNT>;
     cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    k<<<a.S, a.nt, smem, st>>>(a);
+    int per_sm = 0, dev = 0, sms = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, a.nt, smem);
+    const int grid = (int)std::min<long long>((long long)a.S, (long long)std::max(1, per_sm) * sms);
+    if (grid_out) *grid_out = grid;
+    k<<<grid, a.nt, smem, st>>>(a, *q);
     return (int)cudaGetLastError();
 }
 
@@ -607,15 +709,15 @@ size_t round_smem_bytes(int32_t nt, int32_t bpt)
     return s + 2 * (size_t)2 * bpt * nt;  // two row buffers of 2 * n_pad bytes
 }
 
-int launch_round(const RoundArgs &a, cudaStream_t st)
+int launch_round(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q, int *grid_out)
 {
     const size_t smem = round_smem_bytes(a.nt, a.bpt);
     if (a.bpt == 32) {
-        if (a.nt == 32) return launch_variant<32, 32, 32>(a, st, smem);
-        return launch_variant<32, 128, 0>(a, st, smem);  // nt = 64, 96
+        if (a.nt == 32) return launch_variant<32, 32, 32>(a, st, smem, q, grid_out);
+        return launch_variant<32, 128, 0>(a, st, smem, q, grid_out);  // nt = 64, 96
     }
-    if (a.nt == 512) return launch_variant<64, 512, 512>(a, st, smem);  // n_pad = 32768
-    return launch_variant<64, 512, 0>(a, st, smem);
+    if (a.nt == 512) return launch_variant<64, 512, 512>(a, st, smem, q, grid_out);  // n_pad = 32768
+    return launch_variant<64, 512, 0>(a, st, smem, q, grid_out);
 }
 
 }  // namespace absb

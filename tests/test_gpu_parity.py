@@ -266,3 +266,59 @@ def test_full_size_n32768_sampled():
         assert st["E"] == o["E"][i]
         assert (st["D"].astype(np.int64) == o["D"][i]).all()
     assert time.time() - t0 < 600
+
+
+# ---------------------------------------------------------------- asynchronous mode (paper Fig. 5)
+def _replay_async(W, s, L, trace_s, l):
+    """Replay one search of an async run with the targets it actually used."""
+    T = np.array([e[2] for e in trace_s])
+    return oracle.replay_search(W, l, L, T)
+
+
+@pytest.mark.parametrize("n,S,L,steps", [(300, 6, 120, 5), (1500, 4, 300, 3), (64, 6000, 40, 2)])
+def test_async_rounds_replay_bitexact(n, S, L, steps):
+    """Async mode: timing decides which target each round gets, but given the
+    targets a search actually used (trace), its trajectory is determined: the
+    oracle replay must match every (B, E_B), the final state and the hash."""
+    W = random_qubo(n, 40 + n)
+    s = make(W, searches=S, local_flips=L, pool_size=16, seed=3, mode=abs_b200.MODE_ASYNC, trace=True)
+    s.search(steps)
+    tr = s.trace()
+    assert len(tr) == S * steps
+    by = {}
+    for e in tr:
+        by.setdefault(e[0], []).append(e)
+    lad = oracle.default_ladder(n)
+    check = range(S) if S <= 16 else list(range(0, S, 997)) + [S - 1]
+    for i in check:
+        es = sorted(by[i], key=lambda e: e[1])
+        assert [e[1] for e in es] == list(range(steps))
+        rep = _replay_async(W, i, L, es, lad[i % len(lad)])
+        assert (rep["EB"] == np.array([e[4] for e in es])).all()
+        assert all((rep["B"][r] == es[r][3]).all() for r in range(steps))
+        st = s.search_state(i)
+        assert st["hash"] == int(rep["hash"][0]) and st["flips"] == int(rep["flips"][0])
+        assert st["E"] == int(rep["E"][0]) and (st["X"] == rep["X"]).all()
+        assert (st["D"].astype(np.int64) == rep["D"]).all()
+    PX, PE = s.pool(16)
+    assert (np.diff(PE) > 0).all()
+    assert (s.energy(PX) == PE).all()
+    assert PE[0] == min(e[4] for e in tr)
+    st = s.stats()
+    assert st["rounds"] == S * steps
+
+
+def test_async_second_call_continues():
+    n, S, L = 200, 5, 80
+    W = random_qubo(n, 77)
+    s = make(W, searches=S, local_flips=L, pool_size=8, seed=4, mode=abs_b200.MODE_ASYNC, trace=True)
+    s.search(2)
+    s.search(3)
+    tr = s.trace()
+    assert len(tr) == S * 5
+    lad = oracle.default_ladder(n)
+    for i in range(S):
+        es = sorted([e for e in tr if e[0] == i], key=lambda e: e[1])
+        assert [e[1] for e in es] == list(range(5))
+        rep = _replay_async(W, i, L, es, lad[i % len(lad)])
+        assert s.search_state(i)["hash"] == int(rep["hash"][0])
