@@ -141,9 +141,11 @@ ABS_API int abs_seed_pool(abs_ctx *c, const uint32_t *X, int32_t count);
  *     straight search C -> T, L window-policy local flips, emit (B, E_B)
  *     (device Steps 2-5) — then the results are inserted in
  *     search-id order (unless external_merge).
- *   async: the persistent kernel runs until every search has emitted `steps`
- *     more rounds; the host GA thread inserts results and writes new targets
- *     while it runs. */
+ *   async: the persistent kernel runs until steps * searches more rounds
+ *     have been emitted in total; the host GA thread inserts results and
+ *     writes new targets while it runs.  When all searches are
+ *     resident each runs at its own pace (rounds per search may differ);
+ *     otherwise every search does exactly `steps` rounds. */
 ABS_API int abs_search(abs_ctx *c, int64_t steps);
 
 /* Best pool entry (pool[0]): X_out host (words(n) words), *E_out host.

@@ -73,8 +73,9 @@ struct RoundArgs {
 // exchange buffers (mapped pinned host memory, device pointers).
 struct AsyncArgs {
     unsigned long long *queue;  // device: next work item (search, round) = (q % S, base + q / S)
-    long long total;            // items of this launch = S * steps
-    int base;                   // rounds every search had completed before this launch
+    long long total;            // rounds of this launch, all searches together = S * steps
+    int base;                   // shared queue: rounds every search had completed before this launch
+    int owned;                  // 1: CTA b owns search b and draws round tickets (S <= resident CTAs)
     int *done;                  // device [S]: rounds completed per search
     const uint8_t *Tmap;        // mapped [S][2][n_pad/8]: double-buffered targets
     const uint32_t *tseq;       // mapped [S]: latest target version (slot = version & 1)

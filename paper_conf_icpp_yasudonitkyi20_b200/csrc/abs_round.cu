@@ -632,11 +632,14 @@ __device__ __forceinline__ void st_release_gpu(int *p, int v)
 }
 
 // The paper's device loop (Steps 2-5 repeated) as a persistent
-// kernel: CTAs take (search, round) items from a queue, read the search's
-// latest target from mapped host memory (Step 2; a stale target is reused,
-// reading C11), run the round, and publish (B, E_B) to mapped host memory
-// with a system-scope release plus a global counter the host GA polls
-// (P:L408).  Host and device never synchronise directly.
+// kernel.  When every search fits on the GPU (S <= resident CTAs) CTA b owns
+// search b and draws round tickets from a shared budget, so each search runs
+// at its own pace ("each CUDA block operates asynchronously");
+// otherwise CTAs take (search, round) items from a queue.  A round reads the
+// search's latest target from mapped host memory (Step 2; a stale target is
+// reused, reading C11) and publishes (B, E_B) to mapped host memory with a
+// system-scope release plus a global counter the host GA polls.
+// Host and device never synchronise directly.
 template <int kP, int kMaxT, int kNT>
 __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? 32 : (kMaxT == 128 ? 6 : 1))
     round_kernel_async(const RoundArgs A, const AsyncArgs Q)
@@ -648,16 +651,18 @@ __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? 32 : (kMaxT == 128 ? 6 : 
     constexpr bool multi = kMaxT > 32;
     int fbase = 0;
     Round<kP, kMaxT, kNT>::init_barriers(smem);
+    int r_own = Q.owned ? ld_acquire_gpu(Q.done + blockIdx.x) : 0;
     for (;;) {
         if (threadIdx.x == 0) item = (long long)atomicAdd(Q.queue, 1ull);
         if (multi) __syncthreads();
         else __syncwarp();
         const long long q = item;
         if (q >= Q.total) break;
-        const int s = (int)(q % A.S);
-        const int r = Q.base + (int)(q / A.S);
+        const int s = Q.owned ? (int)blockIdx.x : (int)(q % A.S);
+        const int r = Q.owned ? r_own++ : Q.base + (int)(q / A.S);
         if (threadIdx.x == 0) {
-            while (ld_acquire_gpu(Q.done + s) != r) __nanosleep(256);  // round r-1 of s finished
+            if (!Q.owned)
+                while (ld_acquire_gpu(Q.done + s) != r) __nanosleep(256);  // round r-1 of s finished
             // the result slot of round r (double-buffered) must have been consumed by the host
             while ((int)ld_acquire_sys(Q.rack + s) < r - 1) __nanosleep(1024);
             tver = ld_acquire_sys(Q.tseq + s);  // latest published target version
@@ -697,7 +702,9 @@ int launch_variant(const RoundArgs &a, cudaStream_t st, size_t smem, const Async
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, a.nt, smem);
     const int grid = (int)std::min<long long>((long long)a.S, (long long)std::max(1, per_sm) * sms);
     if (grid_out) *grid_out = grid;
-    k<<<grid, a.nt, smem, st>>>(a, *q);
+    AsyncArgs q2 = *q;
+    q2.owned = grid >= a.S ? 1 : 0;
+    k<<<grid, a.nt, smem, st>>>(a, q2);
     return (int)cudaGetLastError();
 }
 

@@ -284,18 +284,21 @@ def test_async_rounds_replay_bitexact(n, S, L, steps):
     s = make(W, searches=S, local_flips=L, pool_size=16, seed=3, mode=abs_b200.MODE_ASYNC, trace=True)
     s.search(steps)
     tr = s.trace()
-    assert len(tr) == S * steps
+    assert len(tr) == S * steps          # rounds per search may differ (searches run freely)
     by = {}
     for e in tr:
         by.setdefault(e[0], []).append(e)
     lad = oracle.default_ladder(n)
     check = range(S) if S <= 16 else list(range(0, S, 997)) + [S - 1]
     for i in check:
-        es = sorted(by[i], key=lambda e: e[1])
-        assert [e[1] for e in es] == list(range(steps))
+        es = sorted(by.get(i, []), key=lambda e: e[1])
+        nr = len(es)
+        assert [e[1] for e in es] == list(range(nr))
+        if nr == 0:
+            continue
         rep = _replay_async(W, i, L, es, lad[i % len(lad)])
         assert (rep["EB"] == np.array([e[4] for e in es])).all()
-        assert all((rep["B"][r] == es[r][3]).all() for r in range(steps))
+        assert all((rep["B"][r] == es[r][3]).all() for r in range(nr))
         st = s.search_state(i)
         assert st["hash"] == int(rep["hash"][0]) and st["flips"] == int(rep["flips"][0])
         assert st["E"] == int(rep["E"][0]) and (st["X"] == rep["X"]).all()
@@ -319,6 +322,8 @@ def test_async_second_call_continues():
     lad = oracle.default_ladder(n)
     for i in range(S):
         es = sorted([e for e in tr if e[0] == i], key=lambda e: e[1])
-        assert [e[1] for e in es] == list(range(5))
+        assert [e[1] for e in es] == list(range(len(es)))
+        if not es:
+            continue
         rep = _replay_async(W, i, L, es, lad[i % len(lad)])
         assert s.search_state(i)["hash"] == int(rep["hash"][0])
