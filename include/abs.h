@@ -201,6 +201,12 @@ ABS_API const char *abs_strerror(int rc);
  * (never NULL; "" if none). */
 ABS_API const char *abs_last_error(void);
 
+/* Diagnostics: per-search, per-warp cycle accounting of the lockstep round
+ * kernel ([searches][32][8] int64: window selection, row wait, row update,
+ * publish/bookkeeping, barrier, tail, flips, straight flips).  Only in a
+ * library built with -DABS_TIMING; otherwise ABS_EINVAL. */
+ABS_API int abs_debug_timing(const abs_ctx *c, long long *out);
+
 /* Library version string. */
 ABS_API const char *abs_version(void);
 

@@ -73,7 +73,7 @@ class abs_stats(C.Structure):
 EXPORTS = [
     "abs_config_init", "abs_create", "abs_create_dev", "abs_seed_pool", "abs_search", "abs_best",
     "abs_stats_get", "abs_pool_get", "abs_pool_insert", "abs_energy", "abs_round_results",
-    "abs_round_targets", "abs_trace_count", "abs_trace_get", "abs_search_state", "abs_destroy", "abs_strerror", "abs_last_error", "abs_version",
+    "abs_round_targets", "abs_trace_count", "abs_trace_get", "abs_search_state", "abs_debug_timing", "abs_destroy", "abs_strerror", "abs_last_error", "abs_version",
 ]
 
 _lib = None
@@ -88,8 +88,8 @@ def load(build_if_missing: bool = True):
     global _lib
     if _lib is not None:
         return _lib
-    path = _build.LIB
-    if build_if_missing:
+    path = os.environ.get("ABS_LIB") or _build.LIB  # ABS_LIB: diagnostics builds only
+    if build_if_missing and not os.environ.get("ABS_LIB"):
         try:
             path = _build.build()
         except Exception as e:  # no nvcc: only an existing library can be used
@@ -114,6 +114,7 @@ def load(build_if_missing: bool = True):
     L.abs_round_results.argtypes = [vp, vp, vp]
     L.abs_round_targets.argtypes = [vp, vp]
     L.abs_trace_count.argtypes = [vp, P(C.c_int64)]
+    L.abs_debug_timing.argtypes = [vp, vp]
     L.abs_trace_get.argtypes = [vp, C.c_int64, P(C.c_int32), P(C.c_int32), vp, vp, P(C.c_int64)]
     L.abs_search_state.argtypes = [vp, C.c_int32, vp, vp, P(C.c_int64), P(C.c_int32), P(C.c_int32),
                                    P(C.c_uint64), P(C.c_int64)]
@@ -283,6 +284,12 @@ class Solver:
         T = np.zeros((self.searches, self.words), np.uint32)
         _check(load().abs_round_targets(self._c, _ptr(T)), "abs_round_targets")
         return T
+
+    def debug_timing(self):
+        """Diagnostics build only: int64 [searches, 32, 8] cycle accumulators."""
+        out = np.zeros((self.searches, 32, 8), np.int64)
+        _check(load().abs_debug_timing(self._c, _ptr(out)), "abs_debug_timing")
+        return out
 
     def trace(self):
         """Async trace: list of (search, round, T, B, E_B) in arrival order."""

@@ -171,6 +171,7 @@ struct abs_ctx {
     std::vector<std::vector<std::vector<uint32_t>>> hist;  // trace: targets by version
     std::vector<TraceEntry> trace;
     int async_grid = 0;
+    long long *timing_d = nullptr;  // diagnostics build
 };
 
 static void free_ctx(abs_ctx *c)
@@ -204,6 +205,7 @@ static void free_ctx(abs_ctx *c)
     if (c->Reb) cudaFreeHost(c->Reb);
     if (c->rcount) cudaFreeHost(c->rcount);
     cudaFree(c->queue_d);
+    cudaFree(c->timing_d);
     cudaFree(c->done_d);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
@@ -420,6 +422,13 @@ static int lockstep_step(abs_ctx *c)
     a.sflips = c->S.sflips;
     a.L = c->L;
     a.S = S;
+#ifdef ABS_TIMING
+    if (!c->timing_d) {
+        ABS_CU(cudaMalloc(&c->timing_d, (size_t)S * 32 * 8 * sizeof(long long)));
+        ABS_CU(cudaMemset(c->timing_d, 0, (size_t)S * 32 * 8 * sizeof(long long)));
+    }
+    a.timing = c->timing_d;
+#endif
     ABS_CU(cudaEventRecord(c->ev0, c->st));
     ABS_CK(launch_round(a, c->st));
     c->launches++;
@@ -825,6 +834,19 @@ int abs_round_targets(const abs_ctx *c, uint32_t *T_out)
     for (int s = 0; s < c->S.S; ++s)
         std::memcpy(T_out + (size_t)s * words, c->T_h + (size_t)s * c->bytes_per_vec, sizeof(uint32_t) * words);
     return ABS_OK;
+}
+
+int abs_debug_timing(const abs_ctx *c, long long *out)
+{
+#ifdef ABS_TIMING
+    if (!c || !out || !c->timing_d) return fail(ABS_ESTATE, "no timing data");
+    ABS_CU(cudaMemcpy(out, c->timing_d, (size_t)c->S.S * 32 * 8 * sizeof(long long), cudaMemcpyDeviceToHost));
+    return ABS_OK;
+#else
+    (void)c;
+    (void)out;
+    return fail(ABS_EINVAL, "built without ABS_TIMING");
+#endif
 }
 
 int abs_trace_count(const abs_ctx *c, int64_t *count)

@@ -67,6 +67,7 @@ struct RoundArgs {
     int64_t *flips, *sflips;
     int64_t L;
     int32_t S;
+    long long *timing;  // diagnostics build only: [S][32][8] cycle accumulators
 };
 
 // Asynchronous mode (ABS_MODE_ASYNC): work queue and the host<->device

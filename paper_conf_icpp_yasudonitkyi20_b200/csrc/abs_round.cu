@@ -43,6 +43,13 @@ constexpr uint64_t kFnvPrime = 0x100000001b3ull;
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWinMax = 256;  // largest l served by the prefetch path (ladder max, reading C7)
 
+// Diagnostics build (-DABS_TIMING): per-warp cycle accounting of the flip loop.
+#ifdef ABS_TIMING
+#define ABS_T(x) x
+#else
+#define ABS_T(x)
+#endif
+
 template <int kP>
 struct MaskOf;
 template <>
@@ -69,6 +76,9 @@ struct RoundSmem {
     long long E, EB, LB;  // E(X), E_B, lower bound on min_i Delta_i(X): thread 0 only
     unsigned long long hash;
     long long nflip, nstraight;
+#ifdef ABS_TIMING
+    long long tacc[32][8];  // [warp][phase] cycles
+#endif
 };
 struct WindowSmem {  // published Delta / x of the next window, by flip parity
     int d[2][kWinMax];
@@ -379,10 +389,12 @@ struct Round {
         if (t == ctl) issue_row(A, k, rowbuf + rowb * (fbase & 1), sm->bar[fbase & 1], nt);
 
         int f = 0;
+        ABS_T(if (lane == 0) for (int q = 0; q < 8; ++q) sm->tacc[warp][q] = 0;)
         for (;; ++f) {
             const int b = (fbase + f) & 1;
             const uint32_t par = (uint32_t)((fbase + f) >> 1) & 1u;
             unsigned char *row = rowbuf + rowb * b;
+            ABS_T(long long tc0 = clock64();)
 
             // ---- window-first selection of the next flip (warp 0), prefetch its row
             if (pre && !straight && left > 1 && warp == nw - 1) {
@@ -447,6 +459,7 @@ struct Round {
                 }
             }
 
+            ABS_T(long long tc1 = clock64(); mbar_wait(&sm->bar[b][0], par); long long tc2 = clock64();)
             // ---- flip k (Alg. 4 lines P:L328-336 / Alg. 5 lines P:L371-376)
             const int c = xk ? -2 : 2;  // 2 phi(x_k), pre-flip bit (Eq.(16))
             {
@@ -465,6 +478,7 @@ struct Round {
                 a += l;  // offset <- (a + l) mod n
                 if (a >= n) a -= n;
             }
+            ABS_T(long long tc3 = clock64();)
             int ci2 = INT_MAX;
             if (!straight) {
                 if (pre) {
@@ -500,6 +514,7 @@ struct Round {
                 }
             }
 
+            ABS_T(long long tc4 = clock64();)
             Red r1;
             if (exact) {
                 r1 = block_reduce(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw);
@@ -508,6 +523,7 @@ struct Round {
                 r1 = Red{INT_MAX, INT_MAX, INT_MAX};
             }
 
+            ABS_T(long long tc5 = clock64();)
             // ---- neighbour tracking (reading C2) and, straight phase, the argmin index
             const bool improve = exact && min(r1.v, 0) < sm->thr[b];  // uniform
             if (t == ctl && exact) {
@@ -545,6 +561,16 @@ struct Round {
                     dk = sv.y;
                     xk = sv.z;
                     exact = sv.w != 0;
+                    ABS_T(if (lane == 0) {
+                        const long long tc6 = clock64();
+                        sm->tacc[warp][0] += tc1 - tc0;
+                        sm->tacc[warp][1] += tc2 - tc1;
+                        sm->tacc[warp][2] += tc3 - tc2;
+                        sm->tacc[warp][3] += tc4 - tc3;
+                        sm->tacc[warp][4] += tc5 - tc4;
+                        sm->tacc[warp][5] += tc6 - tc5;
+                        sm->tacc[warp][6] += 1;
+                    })
                     continue;  // row already in flight
                 }
                 k = r1.i >> 1;
@@ -568,9 +594,23 @@ struct Round {
                 exact = true;
             }
             if (t == ctl) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+            ABS_T(if (lane == 0) {
+                const long long tc6 = clock64();
+                sm->tacc[warp][0] += tc1 - tc0;  // window selection (control warp)
+                sm->tacc[warp][1] += tc2 - tc1;  // wait for the row
+                sm->tacc[warp][2] += tc3 - tc2;  // row update
+                sm->tacc[warp][3] += tc4 - tc3;  // publish + bookkeeping
+                sm->tacc[warp][4] += tc5 - tc4;  // reduction / barrier
+                sm->tacc[warp][5] += tc6 - tc5;  // tracking + next selection
+                sm->tacc[warp][6] += 1;
+                sm->tacc[warp][7] += straight ? 1 : 0;
+            })
         }
 
         fbase += f + 1;  // rows consumed in this round (no row left in flight)
+        ABS_T(if (lane == 0 && A.timing) for (int q = 0; q < 8; ++q)
+                  atomicAdd((unsigned long long *)&A.timing[((size_t)sid * 32 + warp) * 8 + q],
+                            (unsigned long long)sm->tacc[warp][q]);)
 
         // ---- Step 5: store (B, E_B) and the state C' for the next round
         sync();
