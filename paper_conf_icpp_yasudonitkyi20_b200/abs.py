@@ -287,7 +287,7 @@ class Solver:
 
     def debug_timing(self):
         """Diagnostics build only: int64 [searches, 32, 8] cycle accumulators."""
-        out = np.zeros((self.searches, 32, 8), np.int64)
+        out = np.zeros((self.searches, 32, 24), np.int64)
         _check(load().abs_debug_timing(self._c, _ptr(out)), "abs_debug_timing")
         return out
 

@@ -424,8 +424,8 @@ static int lockstep_step(abs_ctx *c)
     a.S = S;
 #ifdef ABS_TIMING
     if (!c->timing_d) {
-        ABS_CU(cudaMalloc(&c->timing_d, (size_t)S * 32 * 8 * sizeof(long long)));
-        ABS_CU(cudaMemset(c->timing_d, 0, (size_t)S * 32 * 8 * sizeof(long long)));
+        ABS_CU(cudaMalloc(&c->timing_d, (size_t)S * 32 * 24 * sizeof(long long)));
+        ABS_CU(cudaMemset(c->timing_d, 0, (size_t)S * 32 * 24 * sizeof(long long)));
     }
     a.timing = c->timing_d;
 #endif
@@ -840,7 +840,7 @@ int abs_debug_timing(const abs_ctx *c, long long *out)
 {
 #ifdef ABS_TIMING
     if (!c || !out || !c->timing_d) return fail(ABS_ESTATE, "no timing data");
-    ABS_CU(cudaMemcpy(out, c->timing_d, (size_t)c->S.S * 32 * 8 * sizeof(long long), cudaMemcpyDeviceToHost));
+    ABS_CU(cudaMemcpy(out, c->timing_d, (size_t)c->S.S * 32 * 24 * sizeof(long long), cudaMemcpyDeviceToHost));
     return ABS_OK;
 #else
     (void)c;

@@ -327,3 +327,20 @@ def test_async_second_call_continues():
             continue
         rep = _replay_async(W, i, L, es, lad[i % len(lad)])
         assert s.search_state(i)["hash"] == int(rep["hash"][0])
+
+
+@pytest.mark.parametrize("n,ladder", [(2000, [256]), (5000, [256, 200]), (10000, [256, 97]), (33, [8])])
+def test_lockstep_large_windows_few_warps(n, ladder):
+    # the window selection is split over min(4, warps) warps; l up to 256
+    W = random_qubo(n, 50)
+    s, o, gB, gEB, gT = run_both(W, 3, 300, 2, pool=8, seed=50, ladder=ladder)
+    assert_same(s, o, gB, gEB, 3, n, 8)
+
+
+@pytest.mark.parametrize("L", [1, 2, 3, 4, 5])
+def test_lockstep_short_local_phases(L):
+    # lookahead pipeline edges: rows / slices issued only for flips that happen
+    n = 3000
+    W = random_qubo(n, 60 + L)
+    s, o, gB, gEB, gT = run_both(W, 4, L, 3, pool=8, seed=60 + L, ladder=[64, 256])
+    assert_same(s, o, gB, gEB, 4, n, 8)
