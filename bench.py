@@ -62,8 +62,13 @@ def make_W(workload: str):
     raise ValueError(workload)
 
 
-def default_searches(workload: str) -> int:
-    return 10000 if workload == "random1k" else 148
+def default_searches(workload: str, n: int, device: int) -> int:
+    """Config 2 fixes 10k searches at n=1024; elsewhere the searches whose
+    CTAs are co-resident on the GPU (148 at n=32k: one 512-thread CTA per SM)."""
+    if workload == "random1k":
+        return 10000
+    import paper_conf_icpp_yasudonitkyi20_b200 as pkg
+    return pkg.device_searches(n, device)
 
 
 # ------------------------------------------------------------------ clocks
@@ -213,7 +218,7 @@ def run_abs(args):
 
     W = make_W(args.workload)
     n = W.shape[0]
-    S = args.searches or default_searches(args.workload)
+    S = args.searches or default_searches(args.workload, n, local)
     L = args.local_flips or n
     Wp = torch.from_numpy(W).pin_memory()
     Wd = Wp.to(f"cuda:{local}", non_blocking=False)

@@ -207,6 +207,12 @@ ABS_API const char *abs_last_error(void);
  * library built with -DABS_TIMING; otherwise ABS_EINVAL. */
 ABS_API int abs_debug_timing(const abs_ctx *c, long long *out);
 
+/* Number of searches whose CTAs are co-resident on `device` for an
+ * n-bit instance (SMs x resident round-kernel CTAs per SM): the search
+ * count that fills the GPU in one wave ("blocks ... run in
+ * parallel").  Needs a visible CUDA device (ABS_ECUDA otherwise). */
+ABS_API int abs_device_searches(int32_t n, int32_t device, int32_t *out);
+
 /* Library version string. */
 ABS_API const char *abs_version(void);
 

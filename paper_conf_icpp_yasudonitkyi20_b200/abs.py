@@ -73,7 +73,7 @@ class abs_stats(C.Structure):
 EXPORTS = [
     "abs_config_init", "abs_create", "abs_create_dev", "abs_seed_pool", "abs_search", "abs_best",
     "abs_stats_get", "abs_pool_get", "abs_pool_insert", "abs_energy", "abs_round_results",
-    "abs_round_targets", "abs_trace_count", "abs_trace_get", "abs_search_state", "abs_debug_timing", "abs_destroy", "abs_strerror", "abs_last_error", "abs_version",
+    "abs_round_targets", "abs_trace_count", "abs_trace_get", "abs_search_state", "abs_debug_timing", "abs_destroy", "abs_strerror", "abs_last_error", "abs_device_searches", "abs_version",
 ]
 
 _lib = None
@@ -124,6 +124,7 @@ def load(build_if_missing: bool = True):
     L.abs_strerror.restype = C.c_char_p
     L.abs_last_error.argtypes = []
     L.abs_last_error.restype = C.c_char_p
+    L.abs_device_searches.argtypes = [C.c_int32, C.c_int32, P(C.c_int32)]
     L.abs_version.argtypes = []
     L.abs_version.restype = C.c_char_p
     for name in EXPORTS:
@@ -312,6 +313,13 @@ class Solver:
         _check(load().abs_search_state(self._c, int(s), _ptr(X), _ptr(D), C.byref(E), C.byref(a), C.byref(l),
                                        C.byref(h), C.byref(f)), "abs_search_state")
         return dict(X=X, D=D, E=int(E.value), a=int(a.value), l=int(l.value), hash=int(h.value), flips=int(f.value))
+
+
+def device_searches(n: int, device: int = 0) -> int:
+    """Searches that fill `device` in one wave for an n-bit instance."""
+    out = C.c_int32()
+    _check(load().abs_device_searches(int(n), int(device), C.byref(out)), "abs_device_searches")
+    return int(out.value)
 
 
 def version() -> str:

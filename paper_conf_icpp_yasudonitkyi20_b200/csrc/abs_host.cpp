@@ -918,6 +918,23 @@ const char *abs_strerror(int rc)
 
 const char *abs_last_error(void) { return g_last_error.c_str(); }
 
+int abs_device_searches(int32_t n, int32_t device, int32_t *out)
+{
+    if (!out || n < 1 || n > 32768) return fail(ABS_EINVAL, "abs_device_searches: n out of range or out == NULL");
+    int prev = 0;
+    ABS_CU(cudaGetDevice(&prev));
+    ABS_CU(cudaSetDevice(device));
+    int n_pad = 0, bpt = 0, nt = 0, per_sm = 0, sms = 0;
+    layout_for(n, n_pad, bpt, nt);
+    const int rc = round_occupancy(nt, bpt, &per_sm);
+    const cudaError_t e2 = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device);
+    cudaSetDevice(prev);
+    ABS_CK(rc);
+    ABS_CU(e2);
+    *out = per_sm * sms;
+    return ABS_OK;
+}
+
 const char *abs_version(void) { return "abs-b200 0.1 (sm_100a)"; }
 
 }  // extern "C"

@@ -101,5 +101,7 @@ int launch_round(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q = nullp
 int launch_batch_init(const Instance &I, const uint8_t *X, int32_t count, int64_t *E, int32_t *delta,
                       cudaStream_t st);
 size_t round_smem_bytes(int32_t nt, int32_t bpt);
+// CTAs of the round kernel for layout (nt, bpt) resident per SM (cudaError_t).
+int round_occupancy(int32_t nt, int32_t bpt, int *per_sm);
 
 }  // namespace absb

@@ -759,6 +759,25 @@ size_t round_smem_bytes(int32_t nt, int32_t bpt)
     return s + 2 * (size_t)2 * bpt * nt;  // two row buffers of 2 * n_pad bytes
 }
 
+template <int kP, int kMaxT, int kNT>
+int occupancy_variant(int nt, size_t smem, int *per_sm)
+{
+    auto k = round_kernel<kP, kMaxT, kNT>;
+    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    return (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k, nt, smem);
+}
+
+int round_occupancy(int32_t nt, int32_t bpt, int *per_sm)
+{
+    const size_t smem = round_smem_bytes(nt, bpt);
+    if (bpt == 32) {
+        if (nt == 32) return occupancy_variant<32, 32, 32>(nt, smem, per_sm);
+        return occupancy_variant<32, 128, 0>(nt, smem, per_sm);
+    }
+    if (nt == 512) return occupancy_variant<64, 512, 512>(nt, smem, per_sm);
+    return occupancy_variant<64, 512, 0>(nt, smem, per_sm);
+}
+
 int launch_round(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q, int *grid_out)
 {
     const size_t smem = round_smem_bytes(a.nt, a.bpt);
