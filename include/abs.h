@@ -202,8 +202,9 @@ ABS_API const char *abs_strerror(int rc);
 ABS_API const char *abs_last_error(void);
 
 /* Diagnostics: per-search, per-warp cycle accounting of the lockstep round
- * kernel ([searches][32][8] int64: window selection, row wait, row update,
- * publish/bookkeeping, barrier, tail, flips, straight flips).  Only in a
+ * kernel ([searches][32][24] int64; [0..5] local flips: window selection,
+ * row wait, row update, publish/bookkeeping, barrier, tail; [6] local flips;
+ * [8..14] the same for straight flips; the rest reserved).  Only in a
  * library built with -DABS_TIMING; otherwise ABS_EINVAL. */
 ABS_API int abs_debug_timing(const abs_ctx *c, long long *out);
 

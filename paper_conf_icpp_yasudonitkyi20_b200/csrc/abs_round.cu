@@ -77,7 +77,7 @@ struct RoundSmem {
     unsigned long long hash;
     long long nflip, nstraight;
 #ifdef ABS_TIMING
-    long long tacc[32][8];  // [warp][phase] cycles
+    long long tacc[32][16];  // [warp][local phases 0-6 | straight phases 8-14] cycles, flips
 #endif
 };
 struct WindowSmem {  // published Delta / x of the next window, by flip parity
@@ -120,28 +120,6 @@ struct Round {
         return ((1u << e1) - 1u) & ~((1u << e0) - 1u);
     }
 
-    // Slots of thread t inside the window {(a + r) mod n : r < l} (Fig. 2).
-    static __device__ __forceinline__ M window_mask(int a, int l, int n, int t, int nt)
-    {
-        const int end = a + l;  // exclusive; > n when the window wraps (reading C6)
-        const int hi1 = min(end, n);
-        const int hi2 = end - n;
-        M cm = 0;
-#pragma unroll
-        for (int j = 0; j < G; ++j) {
-            const int base = 8 * (t + nt * j);
-            const bool h1 = (base + 8 > a) && (base < hi1);
-            const bool h2 = base < hi2;
-            if (h1 | h2) {
-                uint32_t m = 0;
-                if (h1) m |= range8(base, a, hi1);
-                if (h2) m |= range8(base, 0, hi2);
-                cm |= (M)m << (8 * j);
-            }
-        }
-        return cm;
-    }
-
     // Lowest-index argmin over the slots in `cm`; ci2 = 2*index + x (INT_MAX if none).
     static __device__ __forceinline__ void candidates(const int (&g)[kP], M xm, M cm, int t, int nt, int &cv,
                                                       int &ci2)
@@ -154,6 +132,39 @@ struct Round {
             if (bit(cm, s) && d < cv) {
                 cv = d;
                 cs = s;
+            }
+        }
+        ci2 = cs < 0 ? INT_MAX : 2 * slot_index(t, nt, cs) + (int)bit(xm, cs);
+    }
+
+    // candidates() over the window {(a + r) mod n : r < l} (Fig. 2),
+    // visiting only the byte-groups j the window touches (block-uniform) and
+    // skipping a group in warps that own none of its window bits.
+    static __device__ __forceinline__ void candidates_window(const int (&g)[kP], M xm, int a, int l, int n, int t,
+                                                             int nt, int &cv, int &ci2)
+    {
+        const int end = a + l;  // exclusive; > n when the window wraps (reading C6)
+        const int hi1 = min(end, n);
+        const int hi2 = end - n;
+        const int j0 = group_of(a, nt), j1 = group_of(hi1 - 1, nt);
+        const int jw = hi2 > 0 ? group_of(hi2 - 1, nt) : -1;
+        cv = INT_MAX;
+        int cs = -1;
+#pragma unroll
+        for (int j = 0; j < G; ++j) {
+            if ((j < j0 || j > j1) && j > jw) continue;
+            const int base = 8 * (t + nt * j);
+            uint32_t m = 0;
+            if (base + 8 > a && base < hi1) m |= range8(base, a, hi1);
+            if (base < hi2) m |= range8(base, 0, hi2);
+            if (!__any_sync(kFull, m != 0)) continue;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+                const int d = readout(g[8 * j + e], xm, 8 * j + e);
+                if (((m >> e) & 1u) && d < cv) {
+                    cv = d;
+                    cs = 8 * j + e;
+                }
             }
         }
         ci2 = cs < 0 ? INT_MAX : 2 * slot_index(t, nt, cs) + (int)bit(xm, cs);
@@ -373,8 +384,8 @@ struct Round {
         int k, dk, xk;
         {
             int cv, ci2;
-            const M cm = straight ? (M)(xm ^ stm[t]) : window_mask(a, l, n, t, nt);
-            candidates(g, xm, cm, t, nt, cv, ci2);
+            if (straight) candidates(g, xm, (M)(xm ^ stm[t]), t, nt, cv, ci2);
+            else candidates_window(g, xm, a, l, n, t, nt, cv, ci2);
             if (pre && !straight) {
                 int a2 = a + l;
                 if (a2 >= n) a2 -= n;
@@ -389,12 +400,12 @@ struct Round {
         if (t == ctl) issue_row(A, k, rowbuf + rowb * (fbase & 1), sm->bar[fbase & 1], nt);
 
         int f = 0;
-        ABS_T(if (lane == 0) for (int q = 0; q < 8; ++q) sm->tacc[warp][q] = 0;)
+        ABS_T(if (lane == 0) for (int q = 0; q < 16; ++q) sm->tacc[warp][q] = 0;)
         for (;; ++f) {
             const int b = (fbase + f) & 1;
             const uint32_t par = (uint32_t)((fbase + f) >> 1) & 1u;
             unsigned char *row = rowbuf + rowb * b;
-            ABS_T(long long tc0 = clock64();)
+            ABS_T(long long tc0 = clock64(); const int to = straight ? 8 : 0;)
 
             // ---- window-first selection of the next flip (warp 0), prefetch its row
             if (pre && !straight && left > 1 && warp == nw - 1) {
@@ -486,8 +497,7 @@ struct Round {
                     if (a2 >= n) a2 -= n;
                     publish_window(g, xm, a2, l, n, t, nt, win->d[b ^ 1], win->x[b ^ 1]);
                 } else {
-                    const M cm = window_mask(a, l, n, t, nt);
-                    if (__any_sync(kFull, cm != 0)) candidates(g, xm, cm, t, nt, cmin, ci2);
+                    candidates_window(g, xm, a, l, n, t, nt, cmin, ci2);
                 }
             }
 
@@ -563,13 +573,13 @@ struct Round {
                     exact = sv.w != 0;
                     ABS_T(if (lane == 0) {
                         const long long tc6 = clock64();
-                        sm->tacc[warp][0] += tc1 - tc0;
-                        sm->tacc[warp][1] += tc2 - tc1;
-                        sm->tacc[warp][2] += tc3 - tc2;
-                        sm->tacc[warp][3] += tc4 - tc3;
-                        sm->tacc[warp][4] += tc5 - tc4;
-                        sm->tacc[warp][5] += tc6 - tc5;
-                        sm->tacc[warp][6] += 1;
+                        sm->tacc[warp][to + 0] += tc1 - tc0;
+                        sm->tacc[warp][to + 1] += tc2 - tc1;
+                        sm->tacc[warp][to + 2] += tc3 - tc2;
+                        sm->tacc[warp][to + 3] += tc4 - tc3;
+                        sm->tacc[warp][to + 4] += tc5 - tc4;
+                        sm->tacc[warp][to + 5] += tc6 - tc5;
+                        sm->tacc[warp][to + 6] += 1;
                     })
                     continue;  // row already in flight
                 }
@@ -581,7 +591,7 @@ struct Round {
                 straight = false;
                 if (left <= 0) break;
                 int cv, cj;
-                candidates(g, xm, window_mask(a, l, n, t, nt), t, nt, cv, cj);
+                candidates_window(g, xm, a, l, n, t, nt, cv, cj);
                 if (pre) {
                     int a2 = a + l;
                     if (a2 >= n) a2 -= n;
@@ -596,20 +606,19 @@ struct Round {
             if (t == ctl) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
             ABS_T(if (lane == 0) {
                 const long long tc6 = clock64();
-                sm->tacc[warp][0] += tc1 - tc0;  // window selection (control warp)
-                sm->tacc[warp][1] += tc2 - tc1;  // wait for the row
-                sm->tacc[warp][2] += tc3 - tc2;  // row update
-                sm->tacc[warp][3] += tc4 - tc3;  // publish + bookkeeping
-                sm->tacc[warp][4] += tc5 - tc4;  // reduction / barrier
-                sm->tacc[warp][5] += tc6 - tc5;  // tracking + next selection
-                sm->tacc[warp][6] += 1;
-                sm->tacc[warp][7] += straight ? 1 : 0;
+                sm->tacc[warp][to + 0] += tc1 - tc0;  // window selection (control warp)
+                sm->tacc[warp][to + 1] += tc2 - tc1;  // wait for the row
+                sm->tacc[warp][to + 2] += tc3 - tc2;  // row update
+                sm->tacc[warp][to + 3] += tc4 - tc3;  // publish + bookkeeping
+                sm->tacc[warp][to + 4] += tc5 - tc4;  // reduction / barrier
+                sm->tacc[warp][to + 5] += tc6 - tc5;  // tracking + next selection
+                sm->tacc[warp][to + 6] += 1;
             })
         }
 
         fbase += f + 1;  // rows consumed in this round (no row left in flight)
-        ABS_T(if (lane == 0 && A.timing) for (int q = 0; q < 8; ++q)
-                  atomicAdd((unsigned long long *)&A.timing[((size_t)sid * 32 + warp) * 8 + q],
+        ABS_T(if (lane == 0 && A.timing) for (int q = 0; q < 16; ++q)
+                  atomicAdd((unsigned long long *)&A.timing[((size_t)sid * 32 + warp) * 24 + q],
                             (unsigned long long)sm->tacc[warp][q]);)
 
         // ---- Step 5: store (B, E_B) and the state C' for the next round

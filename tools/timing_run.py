@@ -10,8 +10,9 @@ from workloads import random_qubo
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 32768
 lad = [int(x) for x in sys.argv[2].split(",")] if len(sys.argv) > 2 and sys.argv[2] else None
 steps = int(sys.argv[3]) if len(sys.argv) > 3 else 4
+S = int(sys.argv[4]) if len(sys.argv) > 4 else pkg.device_searches(n)
 W = torch.from_numpy(random_qubo(n, 1)).cuda()
-s = pkg.Solver(W, searches=148, local_flips=n, pool_size=64, seed=1, ladder=lad)
+s = pkg.Solver(W, searches=S, local_flips=n, pool_size=64, seed=1, ladder=lad)
 s.search(1)
 t0 = s.debug_timing().astype(np.float64)
 s.search(steps)
@@ -19,20 +20,15 @@ T = s.debug_timing().astype(np.float64) - t0   # steady-state rounds only
 nw = s.stats()["threads_per_search"] // 32
 T = T[:, :nw, :]
 names = ["window", "row_wait", "row_update", "publish_book", "reduce_barrier", "tail"]
-out = {"n": n, "ladder": lad}
+out = {"n": n, "ladder": lad, "searches": S}
 for kind, o in (("local", 0), ("straight", 8)):
     fl = T[:, :, o + 6]
     if fl.sum() == 0:
         continue
     out[kind] = {
         "flips_per_search": float(fl[:, 0].sum() / T.shape[0]),
-        "exact_frac": float(T[:, 0, o + 7].sum() / fl[:, 0].sum()),
-        "row_warps": {nm: round(float(T[:, :-1, o + i].sum() / fl[:, :-1].sum()), 1) for i, nm in enumerate(names)},
+        "row_warps": {nm: round(float(T[:, :-1, o + i].sum() / fl[:, :-1].sum()), 1) for i, nm in enumerate(names)}
+        if nw > 1 else None,
         "control_warp": {nm: round(float(T[:, -1, o + i].sum() / fl[:, -1].sum()), 1) for i, nm in enumerate(names)},
     }
-sub = T[:, -1, 16:24]
-if sub[:, 5].sum() > 0:
-    out["control_selection_subphases"] = {nm: round(float(sub[:, i].sum() / sub[:, 5].sum()), 1) for i, nm in
-                                          enumerate(["wait_row", "part", "bar_sync", "combine_issue", "bookkeeping",
-                                                     "count", "combine_only", "issue_only"]) if nm != "count"}
 print(json.dumps(out, indent=1))
