@@ -8,13 +8,14 @@
 
 namespace absb {
 
-// Every search is held by NT threads (a multiple of 32) with P bits each
-// (P = 32 for n <= 3072, else 64), n_pad = P * NT >= n.  Threads hold their
-// P fields in registers; P = 64 gives 512 threads x 128 registers at n = 32k.
+// Every search is held by NT threads (a multiple of 32) with P bits each,
+// n_pad = P * NT >= n: P = 32 for n <= 1024 (one warp) and n_pad = 3072;
+// P = 64 otherwise (one warp at n_pad = 2048; 512 threads x 128 registers at
+// n = 32k).  Threads hold their P fields in registers.
 inline void layout_for(int n, int &n_pad, int &bpt, int &nt)
 {
     const int p1 = ((n + 1023) / 1024) * 1024;
-    if (p1 <= 3072) {
+    if (p1 == 1024 || p1 == 3072) {
         bpt = 32;
         n_pad = p1;
     } else {

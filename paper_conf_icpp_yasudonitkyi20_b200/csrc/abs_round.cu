@@ -526,7 +526,7 @@ struct Round {
 
             ABS_T(long long tc4 = clock64();)
             Red r1;
-            if (exact) {
+            if (exact || !pre) {  // !pre: the window argmin of the next flip is reduced here too
                 r1 = block_reduce(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw);
             } else {
                 sync();  // row buffer b free; sel[b], thr[b] and the window published
@@ -586,6 +586,14 @@ struct Round {
                 k = r1.i >> 1;
                 xk = r1.i & 1;
                 dk = r1.c;
+                if constexpr (!kMulti) {
+                    // lazy tracking for the next flip, as on the prefetch path: exact only if
+                    // E(X'') + min(0, bound on min Delta(X'')) can beat E_B
+                    __syncwarp();  // lane 0's E / LB / E_B updates of this flip
+                    const long long E1 = sm->E;
+                    const long long LB2 = min(sm->LB - 2 * (long long)A.wmax, -(long long)dk);
+                    exact = E1 + dk + min(LB2, 0LL) < sm->EB;
+                }
             } else if (!sidx) {
                 // X = T: the straight search is over; local search from T (Step 4b)
                 straight = false;
@@ -648,7 +656,7 @@ struct Round {
 };
 
 template <int kP, int kMaxT, int kNT>
-__global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? 32 : (kMaxT == 128 ? 6 : 1)) round_kernel(const RoundArgs A)
+__global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (kMaxT == 128 ? 6 : 1)) round_kernel(const RoundArgs A)
 {
     extern __shared__ __align__(128) unsigned char smem[];
     const int sid = blockIdx.x;
@@ -690,7 +698,7 @@ __device__ __forceinline__ void st_release_gpu(int *p, int v)
 // system-scope release plus a global counter the host GA polls.
 // Host and device never synchronise directly.
 template <int kP, int kMaxT, int kNT>
-__global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? 32 : (kMaxT == 128 ? 6 : 1))
+__global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (kMaxT == 128 ? 6 : 1))
     round_kernel_async(const RoundArgs A, const AsyncArgs Q)
 {
     extern __shared__ __align__(128) unsigned char smem[];
@@ -783,6 +791,7 @@ int round_occupancy(int32_t nt, int32_t bpt, int *per_sm)
         if (nt == 32) return occupancy_variant<32, 32, 32>(nt, smem, per_sm);
         return occupancy_variant<32, 128, 0>(nt, smem, per_sm);
     }
+    if (nt == 32) return occupancy_variant<64, 32, 32>(nt, smem, per_sm);  // n_pad = 2048
     if (nt == 512) return occupancy_variant<64, 512, 512>(nt, smem, per_sm);
     return occupancy_variant<64, 512, 0>(nt, smem, per_sm);
 }
@@ -792,8 +801,9 @@ int launch_round(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q, int *g
     const size_t smem = round_smem_bytes(a.nt, a.bpt);
     if (a.bpt == 32) {
         if (a.nt == 32) return launch_variant<32, 32, 32>(a, st, smem, q, grid_out);
-        return launch_variant<32, 128, 0>(a, st, smem, q, grid_out);  // nt = 64, 96
+        return launch_variant<32, 128, 0>(a, st, smem, q, grid_out);  // nt = 96
     }
+    if (a.nt == 32) return launch_variant<64, 32, 32>(a, st, smem, q, grid_out);  // n_pad = 2048
     if (a.nt == 512) return launch_variant<64, 512, 512>(a, st, smem, q, grid_out);  // n_pad = 32768
     return launch_variant<64, 512, 0>(a, st, smem, q, grid_out);
 }

@@ -128,7 +128,7 @@ def test_config1_n16_bitexact_and_bruteforce():
     (5, 8, 30, 3, 1),          # tiny, ragged word
     (100, 12, 150, 3, 2),      # one warp, ragged
     (1024, 6, 1024, 2, 3),     # config-2 size, one warp, full
-    (1100, 5, 300, 2, 4),      # 2 warps (n_pad 2048), ragged
+    (1100, 5, 300, 2, 4),      # one warp, 64 bits per thread (n_pad 2048), ragged
     (3000, 4, 500, 2, 5),      # 3 warps
     (4100, 3, 400, 2, 6),      # NT = 160
 ])

@@ -6,12 +6,16 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np
 import torch
 import paper_conf_icpp_yasudonitkyi20_b200 as pkg
-from workloads import random_qubo
+from workloads import maxcut_qubo, random_qubo, tsp_qubo
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 32768
+kind = sys.argv[5] if len(sys.argv) > 5 else "random"
 lad = [int(x) for x in sys.argv[2].split(",")] if len(sys.argv) > 2 and sys.argv[2] else None
 steps = int(sys.argv[3]) if len(sys.argv) > 3 else 4
 S = int(sys.argv[4]) if len(sys.argv) > 4 else pkg.device_searches(n)
-W = torch.from_numpy(random_qubo(n, 1)).cuda()
+Wh = {"random": lambda: random_qubo(n, 1), "maxcut": lambda: maxcut_qubo(n, int(round(9.995 * n)), seed=1),
+      "tsp": lambda: tsp_qubo(int(round(n ** 0.5)), seed=1)}[kind]()
+n = Wh.shape[0]
+W = torch.from_numpy(Wh).cuda()
 s = pkg.Solver(W, searches=S, local_flips=n, pool_size=64, seed=1, ladder=lad)
 s.search(1)
 t0 = s.debug_timing().astype(np.float64)
@@ -20,7 +24,7 @@ T = s.debug_timing().astype(np.float64) - t0   # steady-state rounds only
 nw = s.stats()["threads_per_search"] // 32
 T = T[:, :nw, :]
 names = ["window", "row_wait", "row_update", "publish_book", "reduce_barrier", "tail"]
-out = {"n": n, "ladder": lad, "searches": S}
+out = {"n": n, "kind": kind, "ladder": lad, "searches": S}
 for kind, o in (("local", 0), ("straight", 8)):
     fl = T[:, :, o + 6]
     if fl.sum() == 0:
