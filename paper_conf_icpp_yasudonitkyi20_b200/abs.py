@@ -124,10 +124,13 @@ def load(build_if_missing: bool = True):
     L.abs_strerror.restype = C.c_char_p
     L.abs_last_error.argtypes = []
     L.abs_last_error.restype = C.c_char_p
-    L.abs_device_searches.argtypes = [C.c_int32, C.c_int32, P(C.c_int32)]
+    if hasattr(L, "abs_device_searches") or not os.environ.get("ABS_LIB"):  # older diagnostics builds lack it
+        L.abs_device_searches.argtypes = [C.c_int32, C.c_int32, P(C.c_int32)]
     L.abs_version.argtypes = []
     L.abs_version.restype = C.c_char_p
     for name in EXPORTS:
+        if os.environ.get("ABS_LIB") and not hasattr(L, name):
+            continue
         fn = getattr(L, name)
         if fn.restype is C.c_int:  # default restype
             fn.restype = C.c_int

@@ -161,10 +161,12 @@ struct abs_ctx {
     // ---- asynchronous mode (the paper's Fig. 5): mapped pinned exchange buffers
     bool async_ready = false;
     uint8_t *Tmap = nullptr;                     // [S][2][bpv] host view
-    uint32_t *tseq = nullptr, *rtver = nullptr, *rseq = nullptr, *rack = nullptr;
+    uint32_t *tseq = nullptr, *rtver = nullptr, *rack = nullptr;
     uint8_t *Rb = nullptr;                       // [S][2][bpv]
     int64_t *Reb = nullptr;                      // [S][2]
-    unsigned int *rcount = nullptr;
+    unsigned int *rcount_d = nullptr;          // device: results published (ring index)
+    uint32_t *ring = nullptr, *ringseq = nullptr;  // arrival ring [cap][2] / [cap]
+    uint32_t ring_mask = 0, ring_head = 0;
     unsigned long long *queue_d = nullptr;
     int *done_d = nullptr;
     std::vector<uint32_t> tver, consumed;        // host-side per-search versions / consumed rounds
@@ -199,11 +201,12 @@ static void free_ctx(abs_ctx *c)
     if (c->Tmap) cudaFreeHost(c->Tmap);
     if (c->tseq) cudaFreeHost(c->tseq);
     if (c->rtver) cudaFreeHost(c->rtver);
-    if (c->rseq) cudaFreeHost(c->rseq);
     if (c->rack) cudaFreeHost(c->rack);
     if (c->Rb) cudaFreeHost(c->Rb);
     if (c->Reb) cudaFreeHost(c->Reb);
-    if (c->rcount) cudaFreeHost(c->rcount);
+    cudaFree(c->rcount_d);
+    if (c->ring) cudaFreeHost(c->ring);
+    if (c->ringseq) cudaFreeHost(c->ringseq);
     cudaFree(c->queue_d);
     cudaFree(c->timing_d);
     cudaFree(c->done_d);
@@ -476,15 +479,20 @@ static int async_setup(abs_ctx *c)
     ABS_CU(cudaHostAlloc(&c->Reb, (size_t)S * 2 * sizeof(int64_t), fl));
     ABS_CU(cudaHostAlloc(&c->tseq, (size_t)S * sizeof(uint32_t), fl));
     ABS_CU(cudaHostAlloc(&c->rtver, (size_t)S * 2 * sizeof(uint32_t), fl));
-    ABS_CU(cudaHostAlloc(&c->rseq, (size_t)S * sizeof(uint32_t), fl));
     ABS_CU(cudaHostAlloc(&c->rack, (size_t)S * sizeof(uint32_t), fl));
-    ABS_CU(cudaHostAlloc(&c->rcount, sizeof(unsigned int), fl));
     std::memset(c->Tmap, 0, (size_t)S * 2 * bpv);
     std::memset(c->Rb, 0, (size_t)S * 2 * bpv);
     std::memset(c->tseq, 0, (size_t)S * sizeof(uint32_t));
-    std::memset(c->rseq, 0, (size_t)S * sizeof(uint32_t));
     std::memset(c->rack, 0, (size_t)S * sizeof(uint32_t));
-    *c->rcount = 0;
+    ABS_CU(cudaMalloc(&c->rcount_d, sizeof(unsigned int)));
+    ABS_CU(cudaMemset(c->rcount_d, 0, sizeof(unsigned int)));
+    uint32_t cap = 64;
+    while (cap < 2u * (uint32_t)S) cap <<= 1;
+    ABS_CU(cudaHostAlloc(&c->ring, (size_t)cap * 2 * sizeof(uint32_t), fl));
+    ABS_CU(cudaHostAlloc(&c->ringseq, (size_t)cap * sizeof(uint32_t), fl));
+    std::memset(c->ringseq, 0, (size_t)cap * sizeof(uint32_t));
+    c->ring_mask = cap - 1;
+    c->ring_head = 0;
     ABS_CU(cudaMalloc(&c->queue_d, sizeof(unsigned long long)));
     ABS_CU(cudaMalloc(&c->done_d, (size_t)S * sizeof(int)));
     ABS_CU(cudaMemset(c->done_d, 0, (size_t)S * sizeof(int)));
@@ -505,18 +513,36 @@ static int async_setup(abs_ctx *c)
     return ABS_OK;
 }
 
-// Host Steps 2-4 for every result published so far: insert it
-// into the pool, acknowledge the slot, generate one new target for the search.
+// Host Steps 2-4 for every result published so far, in arrival
+// order (the ring): insert it into the pool, acknowledge the slot, generate one
+// new target for the search.  Cost O(results), independent of S.
 static void async_consume(abs_ctx *c)
 {
-    const int S = c->S.S, bpv = c->bytes_per_vec, words = c->pool.words;
+    const int bpv = c->bytes_per_vec, words = c->pool.words;
     std::vector<uint32_t> B(words), T(words);
-    for (int s = 0; s < S; ++s) {
-        const uint32_t rs = vload(c->rseq + s);
-        if (rs <= c->consumed[s]) continue;
+    constexpr uint32_t kBatch = 256;
+    uint32_t es[kBatch], er[kBatch];
+    for (;;) {
+        // collect the arrived entries (sequential reads), then prefetch their result
+        // slots: the slots were written by the GPU, so every first touch is a miss
+        const uint32_t h0 = c->ring_head;
+        uint32_t nb = 0;
+        while (nb < kBatch && vload(c->ringseq + ((h0 + nb) & c->ring_mask)) == h0 + nb + 1u) ++nb;
+        if (nb == 0) break;
         std::atomic_thread_fence(std::memory_order_acquire);
-        while (c->consumed[s] < rs) {
-            const uint32_t r = c->consumed[s];
+        for (uint32_t e = 0; e < nb; ++e) {
+            const uint32_t h = (h0 + e) & c->ring_mask;
+            es[e] = vload(c->ring + 2 * h);
+            er[e] = vload(c->ring + 2 * h + 1);
+            const size_t slot = (size_t)es[e] * 2 + (er[e] & 1);
+            for (int off = 0; off < bpv; off += 64) __builtin_prefetch(c->Rb + slot * bpv + off);
+            __builtin_prefetch(c->Reb + slot);
+            __builtin_prefetch(c->rtver + slot);
+        }
+        c->ring_head = h0 + nb;
+        for (uint32_t e = 0; e < nb; ++e) {
+            const int s = (int)es[e];
+            const uint32_t r = er[e];
             const size_t slot = (size_t)s * 2 + (r & 1);
             std::memcpy(B.data(), c->Rb + slot * bpv, sizeof(uint32_t) * words);
             const int64_t EB = vload(c->Reb + slot);
@@ -562,9 +588,11 @@ static int async_run(abs_ctx *c, int64_t steps)
     q.Rb = (uint8_t *)dev(c->Rb);
     q.Reb = (int64_t *)dev(c->Reb);
     q.rtver = (uint32_t *)dev(c->rtver);
-    q.rseq = (uint32_t *)dev(c->rseq);
     q.rack = (const uint32_t *)dev(c->rack);
-    q.rcount = (unsigned int *)dev(c->rcount);
+    q.rcount = c->rcount_d;
+    q.ring = (uint32_t *)dev(c->ring);
+    q.ringseq = (uint32_t *)dev(c->ringseq);
+    q.ring_mask = c->ring_mask;
     RoundArgs a{};
     a.Wz = c->I.Wz;
     a.wmax = c->I.wmax;
@@ -585,16 +613,22 @@ static int async_run(abs_ctx *c, int64_t steps)
     a.sflips = c->S.sflips;
     a.L = c->L;
     a.S = S;
+#ifdef ABS_TIMING
+    if (!c->timing_d) {
+        ABS_CU(cudaMalloc(&c->timing_d, (size_t)S * 32 * 24 * sizeof(long long)));
+        ABS_CU(cudaMemset(c->timing_d, 0, (size_t)S * 32 * 24 * sizeof(long long)));
+    }
+    a.timing = c->timing_d;
+#endif
 
     // the host GA thread, concurrent with the persistent kernel
     std::atomic<bool> stop{false};
     std::thread ga([c, &stop]() {
-        unsigned int seen = 0;
         for (;;) {
             const bool last = stop.load(std::memory_order_acquire);
-            const unsigned int cnt = vload(c->rcount);  // Step 2: poll the global counter
-            if (cnt != seen || last) {
-                seen = cnt;
+            // Step 2: poll for newly arrived solutions
+            const bool ready = vload(c->ringseq + (c->ring_head & c->ring_mask)) == c->ring_head + 1u;
+            if (ready || last) {
                 async_consume(c);
                 if (last) break;
             } else {

@@ -84,9 +84,11 @@ struct AsyncArgs {
     uint8_t *Rb;                // mapped [S][2][n_pad/8]: B of round r in slot r & 1
     int64_t *Reb;               // mapped [S][2]: E_B
     uint32_t *rtver;            // mapped [S][2]: target version the round used
-    uint32_t *rseq;             // mapped [S]: rounds published
     const uint32_t *rack;       // mapped [S]: rounds consumed by the host
-    unsigned int *rcount;       // mapped: total results published (polled by the host GA)
+    unsigned int *rcount;       // device: total results published; draws the ring index
+    uint32_t *ring;             // mapped [ring_mask + 1][2]: (search, round) in arrival order
+    uint32_t *ringseq;          // mapped [ring_mask + 1]: entry idx valid when ringseq[idx & mask] == idx + 1
+    uint32_t ring_mask;         // capacity - 1; capacity >= 2 S (at most 2 unconsumed results per search)
 };
 
 // Launchers (return cudaError_t as int).

@@ -120,6 +120,28 @@ struct Round {
         return ((1u << e1) - 1u) & ~((1u << e0) - 1u);
     }
 
+    // Slots of thread t inside the window {(a + r) mod n : r < l} (Fig. 2).
+    static __device__ __forceinline__ M window_mask(int a, int l, int n, int t, int nt)
+    {
+        const int end = a + l;  // exclusive; > n when the window wraps (reading C6)
+        const int hi1 = min(end, n);
+        const int hi2 = end - n;
+        M cm = 0;
+#pragma unroll
+        for (int j = 0; j < G; ++j) {
+            const int base = 8 * (t + nt * j);
+            const bool h1 = (base + 8 > a) && (base < hi1);
+            const bool h2 = base < hi2;
+            if (h1 | h2) {
+                uint32_t m = 0;
+                if (h1) m |= range8(base, a, hi1);
+                if (h2) m |= range8(base, 0, hi2);
+                cm |= (M)m << (8 * j);
+            }
+        }
+        return cm;
+    }
+
     // Lowest-index argmin over the slots in `cm`; ci2 = 2*index + x (INT_MAX if none).
     static __device__ __forceinline__ void candidates(const int (&g)[kP], M xm, M cm, int t, int nt, int &cv,
                                                       int &ci2)
@@ -168,6 +190,21 @@ struct Round {
             }
         }
         ci2 = cs < 0 ? INT_MAX : 2 * slot_index(t, nt, cs) + (int)bit(xm, cs);
+    }
+
+    // Window argmin: one warp scans only the window's byte-groups; the
+    // multi-warp kernels keep the mask form (measured faster there, n = 32k).
+    static __device__ __forceinline__ void window_candidates(const int (&g)[kP], M xm, int a, int l, int n, int t,
+                                                             int nt, int &cv, int &ci2)
+    {
+        if constexpr (kMulti) {
+            const M cm = window_mask(a, l, n, t, nt);
+            cv = INT_MAX;
+            ci2 = INT_MAX;
+            if (__any_sync(kFull, cm != 0)) candidates(g, xm, cm, t, nt, cv, ci2);
+        } else {
+            candidates_window(g, xm, a, l, n, t, nt, cv, ci2);
+        }
     }
 
     // 2*index + x of the lowest slot in `cm` whose Delta equals v (INT_MAX if none).
@@ -321,12 +358,15 @@ struct Round {
     }
 
     // ---------------------------------------------------------------- the round
-    // One round of search `sid`: target bits from Ts, (B, E_B) to Bs_out / *EB_out.
+    // One round of search `sid`: target bits from Ts; (B, E_B) go to the
+    // pointers out(Bs, EBp) yields at the end of the round (evaluated late so
+    // that no output address stays live across the flip loop).
     // fbase counts the rows this CTA has consumed before (row buffer and mbarrier
     // phase of flip f are those of use fbase + f); the barriers are initialised
     // once per launch by init_barriers().
+    template <class Out>
     static __device__ __forceinline__ void run(const RoundArgs &A, unsigned char *smem, int sid, const uint8_t *Ts,
-                                               uint8_t *Bs_out, int64_t *EB_out, int &fbase)
+                                               const Out &out, int &fbase)
     {
         const int nt = kNT ? kNT : (kMulti ? A.nt : 32);
         const int n = A.n;
@@ -384,8 +424,13 @@ struct Round {
         int k, dk, xk;
         {
             int cv, ci2;
-            if (straight) candidates(g, xm, (M)(xm ^ stm[t]), t, nt, cv, ci2);
-            else candidates_window(g, xm, a, l, n, t, nt, cv, ci2);
+            if constexpr (kMulti) {  // one inlined scan (code size of the flip loop)
+                const M cm = straight ? (M)(xm ^ stm[t]) : window_mask(a, l, n, t, nt);
+                candidates(g, xm, cm, t, nt, cv, ci2);
+            } else {
+                if (straight) candidates(g, xm, (M)(xm ^ stm[t]), t, nt, cv, ci2);
+                else candidates_window(g, xm, a, l, n, t, nt, cv, ci2);
+            }
             if (pre && !straight) {
                 int a2 = a + l;
                 if (a2 >= n) a2 -= n;
@@ -497,7 +542,7 @@ struct Round {
                     if (a2 >= n) a2 -= n;
                     publish_window(g, xm, a2, l, n, t, nt, win->d[b ^ 1], win->x[b ^ 1]);
                 } else {
-                    candidates_window(g, xm, a, l, n, t, nt, cmin, ci2);
+                    window_candidates(g, xm, a, l, n, t, nt, cmin, ci2);
                 }
             }
 
@@ -526,7 +571,7 @@ struct Round {
 
             ABS_T(long long tc4 = clock64();)
             Red r1;
-            if (exact || !pre) {  // !pre: the window argmin of the next flip is reduced here too
+            if (exact || (!kMulti && !pre)) {  // one warp: the next window argmin is reduced here too
                 r1 = block_reduce(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw);
             } else {
                 sync();  // row buffer b free; sel[b], thr[b] and the window published
@@ -599,7 +644,8 @@ struct Round {
                 straight = false;
                 if (left <= 0) break;
                 int cv, cj;
-                candidates_window(g, xm, a, l, n, t, nt, cv, cj);
+                if constexpr (kMulti) candidates(g, xm, window_mask(a, l, n, t, nt), t, nt, cv, cj);
+                else candidates_window(g, xm, a, l, n, t, nt, cv, cj);
                 if (pre) {
                     int a2 = a + l;
                     if (a2 >= n) a2 -= n;
@@ -637,6 +683,9 @@ struct Round {
             for (int s = 0; s < kP; ++s) gs[(size_t)s * nt + t] = g[s];
             uint8_t *Xs = A.X + (size_t)sid * G * nt;
             const M bm = sbm[t];
+            uint8_t *Bs_out;
+            int64_t *EB_out;
+            out(Bs_out, EB_out);
 #pragma unroll
             for (int j = 0; j < G; ++j) {
                 Xs[t + nt * j] = (uint8_t)(xm >> (8 * j));
@@ -663,7 +712,15 @@ __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (k
     const size_t bpv = (size_t)A.n_pad / 8;
     int fbase = 0;
     Round<kP, kMaxT, kNT>::init_barriers(smem);
-    Round<kP, kMaxT, kNT>::run(A, smem, sid, A.T + sid * bpv, A.B + sid * bpv, A.EB + sid, fbase);
+    uint8_t *const B0 = A.B + sid * bpv;
+    int64_t *const EB0 = A.EB + sid;
+    Round<kP, kMaxT, kNT>::run(
+        A, smem, sid, A.T + sid * bpv,
+        [=](uint8_t *&Bp, int64_t *&EBp) {
+            Bp = B0;
+            EBp = EB0;
+        },
+        fbase);
 }
 
 // ---------------------------------------------------------------- asynchronous mode
@@ -695,49 +752,78 @@ __device__ __forceinline__ void st_release_gpu(int *p, int v)
 // otherwise CTAs take (search, round) items from a queue.  A round reads the
 // search's latest target from mapped host memory (Step 2; a stale target is
 // reused, reading C11) and publishes (B, E_B) to mapped host memory with a
-// system-scope release plus a global counter the host GA polls.
+// system-scope release and appends (search, round) to an arrival ring the host
+// GA polls.
 // Host and device never synchronise directly.
 template <int kP, int kMaxT, int kNT>
 __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (kMaxT == 128 ? 6 : 1))
     round_kernel_async(const RoundArgs A, const AsyncArgs Q)
 {
     extern __shared__ __align__(128) unsigned char smem[];
+    // the current work item, kept in shared memory so that nothing of it stays
+    // live in registers across the flip loop
     __shared__ long long item;
+    __shared__ int cur_s, cur_r, r_own;
     __shared__ uint32_t tver;
     const size_t bpv = (size_t)A.n_pad / 8;
     constexpr bool multi = kMaxT > 32;
     int fbase = 0;
     Round<kP, kMaxT, kNT>::init_barriers(smem);
-    int r_own = Q.owned ? ld_acquire_gpu(Q.done + blockIdx.x) : 0;
+    if (threadIdx.x == 0) r_own = Q.owned ? ld_acquire_gpu(Q.done + blockIdx.x) : 0;
     for (;;) {
-        if (threadIdx.x == 0) item = (long long)atomicAdd(Q.queue, 1ull);
-        if (multi) __syncthreads();
-        else __syncwarp();
-        const long long q = item;
-        if (q >= Q.total) break;
-        const int s = Q.owned ? (int)blockIdx.x : (int)(q % A.S);
-        const int r = Q.owned ? r_own++ : Q.base + (int)(q / A.S);
         if (threadIdx.x == 0) {
-            if (!Q.owned)
-                while (ld_acquire_gpu(Q.done + s) != r) __nanosleep(256);  // round r-1 of s finished
-            // the result slot of round r (double-buffered) must have been consumed by the host
-            while ((int)ld_acquire_sys(Q.rack + s) < r - 1) __nanosleep(1024);
-            tver = ld_acquire_sys(Q.tseq + s);  // latest published target version
+            const long long q = (long long)atomicAdd(Q.queue, 1ull);
+            item = q;
+            if (q < Q.total) {
+                const int s = Q.owned ? (int)blockIdx.x : (int)(q % A.S);
+                const int r = Q.owned ? r_own++ : Q.base + (int)(q / A.S);
+                ABS_T(const long long w0 = clock64();)
+                if (!Q.owned)
+                    while (ld_acquire_gpu(Q.done + s) != r) __nanosleep(256);  // round r-1 of s finished
+                ABS_T(const long long w1 = clock64();)
+                // the result slot of round r (double-buffered) must have been consumed by the host
+                while ((int)ld_acquire_sys(Q.rack + s) < r - 1) __nanosleep(1024);
+                ABS_T(const long long w2 = clock64();)
+                tver = ld_acquire_sys(Q.tseq + s);  // latest published target version
+                cur_s = s;
+                cur_r = r;
+                ABS_T(if (A.timing) {
+                    unsigned long long *tm = (unsigned long long *)&A.timing[((size_t)s * 32) * 24];
+                    atomicAdd(tm + 16, (unsigned long long)(w1 - w0));
+                    atomicAdd(tm + 17, (unsigned long long)(w2 - w1));
+                    atomicAdd(tm + 18, (unsigned long long)(clock64() - w2));
+                    atomicAdd(tm + 20, 1ull);
+                })
+            }
         }
         if (multi) __syncthreads();
         else __syncwarp();
-        const uint32_t v = tver;
-        Round<kP, kMaxT, kNT>::run(A, smem, s, Q.Tmap + ((size_t)s * 2 + (v & 1)) * bpv,
-                                   Q.Rb + ((size_t)s * 2 + (r & 1)) * bpv, Q.Reb + (size_t)s * 2 + (r & 1), fbase);
-        __threadfence_system();
+        if (item >= Q.total) break;
+        Round<kP, kMaxT, kNT>::run(
+            A, smem, cur_s, Q.Tmap + ((size_t)cur_s * 2 + (tver & 1)) * bpv,
+            [&](uint8_t *&Bp, int64_t *&EBp) {
+                const int s = cur_s, r = cur_r;
+                Bp = Q.Rb + ((size_t)s * 2 + (r & 1)) * bpv;
+                EBp = Q.Reb + (size_t)s * 2 + (r & 1);
+            },
+            fbase);
+        if (threadIdx.x == 0) Q.rtver[(size_t)cur_s * 2 + (cur_r & 1)] = tver;
+        __threadfence_system();  // B, E_B and the target version reach host memory ...
         if (multi) __syncthreads();
         else __syncwarp();
         if (threadIdx.x == 0) {
-            Q.rtver[(size_t)s * 2 + (r & 1)] = v;
-            __threadfence_system();
-            st_release_sys(Q.rseq + s, (uint32_t)(r + 1));
-            atomicAdd_system(Q.rcount, 1u);
+            ABS_T(const long long p0 = clock64();)
+            const int s = cur_s, r = cur_r;
+            // arrival ring: the host GA drains results in this order.  The
+            // index comes from a DEVICE counter: a system-scope atomic on host memory
+            // serialises every CTA over PCIe (~1M results/s for the whole GPU)
+            const uint32_t idx = atomicAdd(Q.rcount, 1u);
+            Q.ring[2 * (idx & Q.ring_mask)] = (uint32_t)s;
+            Q.ring[2 * (idx & Q.ring_mask) + 1] = (uint32_t)r;
+            st_release_sys(Q.ringseq + (idx & Q.ring_mask), idx + 1u);  // ... before the ring entry
             st_release_gpu(Q.done + s, r + 1);
+            ABS_T(if (A.timing) atomicAdd((unsigned long long *)&A.timing[((size_t)s * 32) * 24 + 19],
+                                          (unsigned long long)(clock64() - p0));)
         }
     }
 }
