@@ -299,6 +299,19 @@ def run_abs(args):
             "algorithmic_bytes_per_launch": flips * 2.0 * n / max(1, launches),
             "avg_launch_ms": 1e3 * kern_s / max(1, launches),
             "kernel_share_of_step": kern_s / (ms * 1e-3) if ms > 0 else None}
+    n_pad = int(st1["n_pad"])
+    if 2 * n_pad * n_pad <= 126 * 2 ** 20:
+        # W is L2-resident (n <= ~8k): the second roof of SURVEY §8(d) binds, n int32
+        # adds per flip against the INT32 pipe: 64 lanes/clk/SM (IMAD/IADD3 issue
+        # every 2 cycles per SMSP, B300_MICROARCH "pipe rates") x SMs x max SM clock
+        sms = torch.cuda.get_device_properties(local).multi_processor_count
+        mhz = float(peaks.get("sm_max_mhz", 1965.0))
+        int_peak = sms * 64 * mhz * 1e6 / 1e12
+        ach = flips * float(n) / kern_s / 1e12 if kern_s > 0 else None
+        roof.update({"bound": "alu", "achieved": ach, "peak": int_peak, "unit": "T int32 adds/s",
+                     "frac": (ach / int_peak) if ach else None,
+                     "peak_source": "derived: %d SMs x 64 int32 lanes/clk x %.0f MHz" % (sms, mhz),
+                     "row_bytes_GBps": achieved})
     solver.close()
     del solver
     torch.cuda.synchronize()
