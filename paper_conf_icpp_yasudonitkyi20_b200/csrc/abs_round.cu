@@ -77,7 +77,7 @@ struct RoundSmem {
     unsigned long long hash;
     long long nflip, nstraight;
 #ifdef ABS_TIMING
-    long long tacc[32][16];  // [warp][local phases 0-6 | straight phases 8-14] cycles, flips
+    long long tacc[32][24];  // [warp][local 0-6 | straight 8-14 | selection sub-phases 16-20]
 #endif
 };
 struct WindowSmem {  // published Delta / x of the next window, by flip parity
@@ -445,7 +445,7 @@ struct Round {
         if (t == ctl) issue_row(A, k, rowbuf + rowb * (fbase & 1), sm->bar[fbase & 1], nt);
 
         int f = 0;
-        ABS_T(if (lane == 0) for (int q = 0; q < 16; ++q) sm->tacc[warp][q] = 0;)
+        ABS_T(if (lane == 0) for (int q = 0; q < 24; ++q) sm->tacc[warp][q] = 0;)
         for (;; ++f) {
             const int b = (fbase + f) & 1;
             const uint32_t par = (uint32_t)((fbase + f) >> 1) & 1u;
@@ -464,13 +464,18 @@ struct Round {
                     if (end >= n || h0 == 0) mbar_wait(&sm->bar[b][0], par);
                     if (h1 == 1) mbar_wait(&sm->bar[b][1], par);
                 }
+                ABS_T(const long long ts1 = clock64();)
                 const int *wd = win->d[b];
                 const uint8_t *wx = win->x[b];
                 const short *rw = reinterpret_cast<const short *>(row);
-                int bv = INT_MAX, bi = INT_MAX, bx = 0;
-                // l <= kWinMax = 8 * 32: a lane's loads are issued in two batches of four
+                // key = (Delta_i(X_{f+1}) << 32) | (2i + x_i): its minimum is the
+                // lowest-index argmin (reading C5) and carries x_i along
+                long long best = LLONG_MAX;
+                // l <= kWinMax = 8 * 32: a lane's loads are issued in batches of four;
+                // batches wholly beyond l are skipped (warp-uniform)
 #pragma unroll
                 for (int h = 0; h < kWinMax / 128; ++h) {
+                    if (h > 0 && 128 * h >= l) break;
                     int dd[4], ww[4], xx[4], ii[4];
 #pragma unroll
                     for (int q = 0; q < 4; ++q) {
@@ -491,28 +496,32 @@ struct Round {
                     for (int q = 0; q < 4; ++q) {
                         if (lane + 32 * (4 * h + q) < l) {
                             const int i = ii[q];
-                            int d = dd[q];
-                            int xn = xx[q];
-                            if (i == k) {
-                                d = -d;  // Eq.(6), k = i
-                                xn ^= 1;
-                            } else {
-                                d += (xx[q] == xk) ? 2 * ww[q] : -2 * ww[q];  // Eq.(16)
-                            }
-                            if (d < bv || (d == bv && i < bi)) {
-                                bv = d;
-                                bi = i;
-                                bx = xn;
-                            }
+                            const bool isk = i == k;
+                            const int w2 = (xx[q] == xk) ? 2 * ww[q] : -2 * ww[q];  // Eq.(16)
+                            const int d = isk ? -dd[q] : dd[q] + w2;                  // Eq.(6) at i = k
+                            const int xn = xx[q] ^ (int)isk;
+                            best = min(best, (long long)(((unsigned long long)(unsigned)d << 32) |
+                                                         (unsigned)(2 * i + xn)));
                         }
                     }
                 }
+                const int bv = (int)(best >> 32);
+                ABS_T(const long long ts2 = clock64();)
                 const int mv = __reduce_min_sync(kFull, bv);
-                const int mi = __reduce_min_sync(kFull, bv == mv ? 2 * bi + bx : INT_MAX);
+                const int mi = __reduce_min_sync(kFull, bv == mv ? (int)(unsigned)best : INT_MAX);
+                ABS_T(const long long ts3 = clock64();)
                 if (lane == 0) {
                     issue_row(A, mi >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
                     sm->sel[b] = make_int4(mi >> 1, mv, mi & 1, 1);
                 }
+                ABS_T(if (lane == 0) {
+                    const long long ts4 = clock64();
+                    sm->tacc[warp][16] += ts1 - tc0;  // wait for row k_f's window half
+                    sm->tacc[warp][17] += ts2 - ts1;  // window arithmetic
+                    sm->tacc[warp][18] += ts3 - ts2;  // two warp reductions
+                    sm->tacc[warp][19] += ts4 - ts3;  // TMA issue + sel
+                    sm->tacc[warp][20] += 1;
+                })
             }
 
             ABS_T(long long tc1 = clock64(); mbar_wait(&sm->bar[b][0], par); long long tc2 = clock64();)
@@ -671,7 +680,7 @@ struct Round {
         }
 
         fbase += f + 1;  // rows consumed in this round (no row left in flight)
-        ABS_T(if (lane == 0 && A.timing) for (int q = 0; q < 16; ++q)
+        ABS_T(if (lane == 0 && A.timing) for (int q = 0; q < 24; ++q)
                   atomicAdd((unsigned long long *)&A.timing[((size_t)sid * 32 + warp) * 24 + q],
                             (unsigned long long)sm->tacc[warp][q]);)
 

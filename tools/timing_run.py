@@ -35,4 +35,8 @@ for kind, o in (("local", 0), ("straight", 8)):
         if nw > 1 else None,
         "control_warp": {nm: round(float(T[:, -1, o + i].sum() / fl[:, -1].sum()), 1) for i, nm in enumerate(names)},
     }
+sub = T[:, -1, 16:21]
+if sub[:, 4].sum() > 0:
+    out["selection_subphases"] = {nm: round(float(sub[:, i].sum() / sub[:, 4].sum()), 1) for i, nm in
+                                  enumerate(["wait_row_half", "arith", "reduce", "issue"])}
 print(json.dumps(out, indent=1))
