@@ -41,7 +41,11 @@ namespace {
 
 constexpr uint64_t kFnvPrime = 0x100000001b3ull;
 constexpr unsigned kFull = 0xffffffffu;
-constexpr int kWinMax = 256;  // largest l served by the prefetch path (ladder max, reading C7)
+constexpr int kWinMax = 256;
+#ifndef ABS_ROW_CHUNKS
+#define ABS_ROW_CHUNKS 1
+#endif
+constexpr int kRowChunks = ABS_ROW_CHUNKS;  // bulk copies (and mbarriers) per W row: 1 or 2  // largest l served by the prefetch path (ladder max, reading C7)
 
 // Diagnostics build (-DABS_TIMING): per-warp cycle accounting of the flip loop.
 #ifdef ABS_TIMING
@@ -274,7 +278,7 @@ struct Round {
         cmin = INT_MAX;
 #pragma unroll
         for (int j = 0; j < G; ++j) {
-            if (j % (G / 2) == 0) mbar_wait(&bars[j / (G / 2)], par);
+            if (kRowChunks == 2 ? (j % (G / 2) == 0) : (j == 0)) mbar_wait(&bars[kRowChunks == 2 ? j / (G / 2) : 0], par);
             const uint4 w4 = row4[t + nt * j];
             const uint32_t wv[4] = {w4.x, w4.y, w4.z, w4.w};
 #pragma unroll
@@ -303,8 +307,15 @@ struct Round {
         const char *src = reinterpret_cast<const char *>(A.Wz) + (size_t)k * (size_t)A.n_pad * 2;
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
-            mbar_arrive_expect_tx(&bars[h], half);
-            bulk_g2s(buf + (size_t)half * h, src + (size_t)half * h, half, &bars[h]);
+            if (kRowChunks == 1) {
+                if (h == 0) {
+                    mbar_arrive_expect_tx(&bars[0], 2 * half);
+                    bulk_g2s(buf, src, 2 * half, &bars[0]);
+                }
+            } else {
+                mbar_arrive_expect_tx(&bars[h], half);
+                bulk_g2s(buf + (size_t)half * h, src + (size_t)half * h, half, &bars[h]);
+            }
         }
     }
 
@@ -461,8 +472,12 @@ struct Round {
                     const int end = a1 + l - 1;
                     const int h0 = group_of(a1, nt) / (G / 2);
                     const int h1 = (end >= n) ? 1 : group_of(end, nt) / (G / 2);
-                    if (end >= n || h0 == 0) mbar_wait(&sm->bar[b][0], par);
-                    if (h1 == 1) mbar_wait(&sm->bar[b][1], par);
+                    if (kRowChunks == 1) {
+                        mbar_wait(&sm->bar[b][0], par);
+                    } else {
+                        if (end >= n || h0 == 0) mbar_wait(&sm->bar[b][0], par);
+                        if (h1 == 1) mbar_wait(&sm->bar[b][1], par);
+                    }
                 }
                 ABS_T(const long long ts1 = clock64();)
                 const int *wd = win->d[b];
