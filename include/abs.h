@@ -208,6 +208,23 @@ ABS_API const char *abs_last_error(void);
  * library built with -DABS_TIMING; otherwise ABS_EINVAL. */
 ABS_API int abs_debug_timing(const abs_ctx *c, long long *out);
 
+/* Ising front end.  The Ising Hamiltonian
+ *     H(S) = -sum_{i<j} J_ij s_i s_j - sum_i h_i s_i,   s_i in {-1,+1}
+ * maps to a QUBO (each bit is a spin, value 0/1 instead of -1/+1) by
+ * s_i = 2 x_i - 1, so that H(S) = E(X) + offset with E of Eq.(1):
+ *     W_ij = -2 J_ij (i != j),  W_ii = 2 sum_{j!=i} J_ij - 2 h_i,
+ *     offset = sum_i h_i - sum_{i<j} J_ij.
+ * Host-only (no GPU).  J: n x n int32 row-major, only i < j is read (J_ij for
+ * the pair); h: n int32.  W_out: n x n int16 (symmetric), *offset_out int64.
+ * ABS_ERANGE if some W entry leaves int16; ABS_EINVAL for bad arguments. */
+ABS_API int abs_ising_to_qubo(int32_t n, const int32_t *J, const int32_t *h, int16_t *W_out, int64_t *offset_out);
+
+/* Inverse map, exact in integers: J2_out = 2 J (n x n, zero diagonal,
+ * symmetric), h2_out = 2 h (n), *offset2_out = 2 * offset, with
+ * J_ij = -W_ij / 2, h_i = -(sum_j W_ij) / 2, offset = sum h - sum_{i<j} J.
+ * Host-only.  Any output may be NULL. */
+ABS_API int abs_qubo_to_ising(int32_t n, const int16_t *W, int32_t *J2_out, int32_t *h2_out, int64_t *offset2_out);
+
 /* Number of searches whose CTAs are co-resident on `device` for an
  * n-bit instance (SMs x resident round-kernel CTAs per SM): the search
  * count that fills the GPU in one wave ("blocks ... run in

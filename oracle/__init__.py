@@ -63,6 +63,8 @@ def lib():
         L.oracle_philox4x32_10.argtypes = [_P(C.c_uint32), _P(C.c_uint32), _P(C.c_uint32)]
         L.oracle_energy.restype = C.c_int64
         L.oracle_energy.argtypes = [C.c_int32, _P(C.c_int16), _P(C.c_uint32)]
+        L.oracle_ising_energy.restype = C.c_int64
+        L.oracle_ising_energy.argtypes = [C.c_int32, _P(C.c_int32), _P(C.c_int32), _P(C.c_int8)]
         L.oracle_delta_by_definition.restype = C.c_int64
         L.oracle_delta_by_definition.argtypes = [C.c_int32, _P(C.c_int16), _P(C.c_uint32), C.c_int32]
         L.oracle_init_batch.argtypes = [C.c_int32, _P(C.c_int16), C.c_int32, _P(C.c_uint32), _P(C.c_int64), _P(C.c_int64)]
@@ -117,6 +119,14 @@ def energy(W, X) -> int:
     W = _W(W)
     X = _X(X, W.shape[0])
     return int(lib().oracle_energy(W.shape[0], _ptr(W, C.c_int16), _ptr(X, C.c_uint32)))
+
+
+def ising_energy(J, h, s) -> int:
+    """P:L40 for spins s in {-1,+1} (pairs i<j, reading E1)."""
+    J = np.ascontiguousarray(J, dtype=np.int32)
+    h = np.ascontiguousarray(h, dtype=np.int32)
+    s = np.ascontiguousarray(s, dtype=np.int8)
+    return int(lib().oracle_ising_energy(J.shape[0], _ptr(J, C.c_int32), _ptr(h, C.c_int32), _ptr(s, C.c_int8)))
 
 
 def delta_by_definition(W, X, k: int) -> int:

@@ -73,7 +73,7 @@ class abs_stats(C.Structure):
 EXPORTS = [
     "abs_config_init", "abs_create", "abs_create_dev", "abs_seed_pool", "abs_search", "abs_best",
     "abs_stats_get", "abs_pool_get", "abs_pool_insert", "abs_energy", "abs_round_results",
-    "abs_round_targets", "abs_trace_count", "abs_trace_get", "abs_search_state", "abs_debug_timing", "abs_destroy", "abs_strerror", "abs_last_error", "abs_device_searches", "abs_version",
+    "abs_round_targets", "abs_trace_count", "abs_trace_get", "abs_search_state", "abs_debug_timing", "abs_destroy", "abs_strerror", "abs_last_error", "abs_device_searches", "abs_ising_to_qubo", "abs_qubo_to_ising", "abs_version",
 ]
 
 _lib = None
@@ -126,6 +126,9 @@ def load(build_if_missing: bool = True):
     L.abs_last_error.restype = C.c_char_p
     if hasattr(L, "abs_device_searches") or not os.environ.get("ABS_LIB"):  # older diagnostics builds lack it
         L.abs_device_searches.argtypes = [C.c_int32, C.c_int32, P(C.c_int32)]
+    if hasattr(L, "abs_ising_to_qubo") or not os.environ.get("ABS_LIB"):
+        L.abs_ising_to_qubo.argtypes = [C.c_int32, vp, vp, vp, P(C.c_int64)]
+        L.abs_qubo_to_ising.argtypes = [C.c_int32, vp, vp, vp, P(C.c_int64)]
     L.abs_version.argtypes = []
     L.abs_version.restype = C.c_char_p
     for name in EXPORTS:
@@ -316,6 +319,32 @@ class Solver:
         _check(load().abs_search_state(self._c, int(s), _ptr(X), _ptr(D), C.byref(E), C.byref(a), C.byref(l),
                                        C.byref(h), C.byref(f)), "abs_search_state")
         return dict(X=X, D=D, E=int(E.value), a=int(a.value), l=int(l.value), hash=int(h.value), flips=int(f.value))
+
+
+def ising_to_qubo(J, h):
+    """Ising (J, h) of P:L40 -> (W int16 [n, n], offset) with H(S) = E(X) + offset,
+    s_i = 2 x_i - 1.  Only the upper triangle of J is read."""
+    J = np.ascontiguousarray(J, dtype=np.int32)
+    h = np.ascontiguousarray(h, dtype=np.int32)
+    n = h.shape[0]
+    if J.shape != (n, n):
+        raise ValueError("J must be n x n")
+    W = np.zeros((n, n), np.int16)
+    off = C.c_int64()
+    _check(load().abs_ising_to_qubo(n, _ptr(J), _ptr(h), _ptr(W), C.byref(off)), "abs_ising_to_qubo")
+    return W, int(off.value)
+
+
+def qubo_to_ising(W):
+    """W -> (2J, 2h, 2*offset) exactly (integers): the Ising form of Eq.(1)
+    with H(S) = E(X) + offset."""
+    W = np.ascontiguousarray(W, dtype=np.int16)
+    n = W.shape[0]
+    J2 = np.zeros((n, n), np.int32)
+    h2 = np.zeros(n, np.int32)
+    off2 = C.c_int64()
+    _check(load().abs_qubo_to_ising(n, _ptr(W), _ptr(J2), _ptr(h2), C.byref(off2)), "abs_qubo_to_ising")
+    return J2, h2, int(off2.value)
 
 
 def device_searches(n: int, device: int = 0) -> int:

@@ -952,6 +952,56 @@ const char *abs_strerror(int rc)
 
 const char *abs_last_error(void) { return g_last_error.c_str(); }
 
+int abs_ising_to_qubo(int32_t n, const int32_t *J, const int32_t *h, int16_t *W_out, int64_t *offset_out)
+{
+    if (n < 1 || !J || !h || !W_out || !offset_out) return fail(ABS_EINVAL, "abs_ising_to_qubo: bad arguments");
+    // s_i = 2 x_i - 1: -J s_i s_j = -4J x_i x_j + 2J (x_i + x_j) - J;  -h s_i = -2h x_i + h
+    int64_t offset = 0;
+    std::vector<int64_t> lin((size_t)n, 0);
+    for (int32_t i = 0; i < n; ++i) {
+        lin[i] -= 2 * (int64_t)h[i];
+        offset += h[i];
+        for (int32_t j = i + 1; j < n; ++j) {
+            const int64_t Jij = J[(size_t)i * n + j];
+            lin[i] += 2 * Jij;
+            lin[j] += 2 * Jij;
+            offset -= Jij;
+        }
+    }
+    for (int32_t i = 0; i < n; ++i) {
+        for (int32_t j = 0; j < n; ++j) {
+            // x^T W x counts the pair (i, j) twice: W_ij = -4 J / 2
+            const int64_t v = i == j ? lin[i] : -2 * (int64_t)J[(size_t)std::min(i, j) * n + std::max(i, j)];
+            if (v < INT16_MIN || v > INT16_MAX)
+                return fail(ABS_ERANGE, "abs_ising_to_qubo: W entry out of int16 range at (" + std::to_string(i) +
+                                            ", " + std::to_string(j) + ")");
+            W_out[(size_t)i * n + j] = (int16_t)v;
+        }
+    }
+    *offset_out = offset;
+    return ABS_OK;
+}
+
+int abs_qubo_to_ising(int32_t n, const int16_t *W, int32_t *J2_out, int32_t *h2_out, int64_t *offset2_out)
+{
+    if (n < 1 || !W) return fail(ABS_EINVAL, "abs_qubo_to_ising: bad arguments");
+    int64_t off2 = 0;
+    for (int32_t i = 0; i < n; ++i) {
+        int64_t row = 0;
+        for (int32_t j = 0; j < n; ++j) {
+            const int64_t w = W[(size_t)i * n + j];
+            if (w != W[(size_t)j * n + i]) return fail(ABS_EINVAL, "abs_qubo_to_ising: W is not symmetric");
+            row += w;
+            if (J2_out) J2_out[(size_t)i * n + j] = i == j ? 0 : (int32_t)(-w);
+            if (j > i) off2 += w;  // -sum_{i<j} 2J = +sum_{i<j} W_ij
+        }
+        if (h2_out) h2_out[i] = (int32_t)(-row);
+        off2 -= row;  // sum 2h = -sum_i sum_j W_ij
+    }
+    if (offset2_out) *offset2_out = off2;
+    return ABS_OK;
+}
+
 int abs_device_searches(int32_t n, int32_t device, int32_t *out)
 {
     if (!out || n < 1 || n > 32768) return fail(ABS_EINVAL, "abs_device_searches: n out of range or out == NULL");
