@@ -49,6 +49,10 @@ class _Cfg(C.Structure):
         ("p_cross", C.c_int32),
         ("p_mut", C.c_int32),
         ("mut_max", C.c_int32),
+        ("policy", C.c_int32),
+        ("sa_tau_min", C.c_int32),
+        ("sa_tau_max", C.c_int32),
+        ("sa_levels", C.c_int32),
     ]
 
 
@@ -77,6 +81,10 @@ def lib():
         L.oracle_replay_search.argtypes = [C.c_int32, _P(C.c_int16), C.c_int32, C.c_int64, C.c_int32,
                                            _P(C.c_uint32), _P(C.c_uint32), _P(C.c_int64), _P(C.c_int64),
                                            _P(C.c_int32), _P(C.c_uint64), _P(C.c_int64), _P(C.c_uint32), _P(C.c_int64)]
+        L.oracle_sa_threshold.restype = C.c_uint64
+        L.oracle_sa_threshold.argtypes = [C.c_int64, C.c_int32]
+        L.oracle_local_sa.restype = None
+        L.oracle_local_sa.argtypes = [_P(_Search), C.c_int64]
         L.oracle_bruteforce.restype = C.c_int64
         L.oracle_bruteforce.argtypes = [C.c_int32, _P(C.c_int16), _P(C.c_uint32)]
         L.oracle_pool_insert.restype = C.c_int
@@ -155,6 +163,11 @@ def bruteforce(W):
 
 
 # ---------------------------------------------------------------- runs
+def sa_threshold(dE: int, tau: int) -> int:
+    """Reading E2: the uint32 acceptance bound of an uphill move dE > 0."""
+    return int(lib().oracle_sa_threshold(int(dE), int(tau)))
+
+
 def default_ladder(n: int):
     """Reading C7: l in {4, 8, 16, ..., min(256, n/4)} (n < 16 -> {max(1, n//4)})."""
     top = min(256, max(1, n // 4))
@@ -177,6 +190,10 @@ class Config:
     p_cross: int = 450
     p_mut: int = 450
     mut_max: int | None = None        # default max(1, n // 32)
+    policy: int = 0                   # 0 = window (Fig. 2), 1 = SA (Eq.(7), reading E2)
+    sa_tau_min: int = 1
+    sa_tau_max: int = 1
+    sa_levels: int = 1
 
     def c(self) -> _Cfg:
         c = _Cfg()
@@ -193,6 +210,10 @@ class Config:
         c.p_cross = self.p_cross
         c.p_mut = self.p_mut
         c.mut_max = max(1, self.n // 32) if self.mut_max is None else int(self.mut_max)
+        c.policy = int(self.policy)
+        c.sa_tau_min = int(self.sa_tau_min)
+        c.sa_tau_max = int(self.sa_tau_max)
+        c.sa_levels = int(self.sa_levels)
         return c
 
 
@@ -246,6 +267,8 @@ class _Search(C.Structure):
         ("n", C.c_int32), ("W", _P(C.c_int16)), ("x", _P(C.c_uint32)), ("d", _P(C.c_int64)),
         ("E", C.c_int64), ("a", C.c_int32), ("l", C.c_int32), ("b", _P(C.c_uint32)),
         ("EB", C.c_int64), ("hash", C.c_uint64), ("flips", C.c_int64), ("overflow", C.c_int32),
+        ("policy", C.c_int32), ("tau", C.c_int32), ("sid", C.c_uint32), ("seed", C.c_uint64),
+        ("sa_ctr", C.c_uint64),
     ]
 
 
@@ -309,6 +332,21 @@ class Search:
 
     def local(self, L: int):
         lib().oracle_local(C.byref(self._s), C.c_int64(int(L)))
+
+    def set_sa(self, tau: int, sid: int = 0, seed: int = 1, ctr: int = 0):
+        """Switch this search to the SA policy (reading E2)."""
+        self._s.policy = 1
+        self._s.tau = int(tau)
+        self._s.sid = int(sid)
+        self._s.seed = int(seed) & 0xFFFFFFFFFFFFFFFF
+        self._s.sa_ctr = int(ctr)
+
+    @property
+    def sa_ctr(self) -> int:
+        return int(self._s.sa_ctr)
+
+    def local_sa(self, L: int):
+        lib().oracle_local_sa(C.byref(self._s), C.c_int64(int(L)))
 
     def round(self, T, L: int):
         T = np.ascontiguousarray(T, dtype=np.uint32)
