@@ -64,6 +64,17 @@ extern "C" {
                              * targets and results through pinned buffers
                              * without synchronising. */
 
+/* Local-search policies ("any policy, including a greedy algorithm
+ * and SA"; reading E2). */
+#define ABS_POLICY_WINDOW 0 /* Fig. 2 / P:L305: argmin over a sliding window of l bits */
+#define ABS_POLICY_SA 1     /* Eq.(7) / Alg. 1: random bit, accepted if dE <= 0, else
+                             * with p = 2^(-dE/tau) (linear between integer exponents);
+                             * proposals from Philox4x32-10, key = seed, counter =
+                             * (lo32(c), hi32(c), global search id, 'SAPL'), c = the
+                             * search's proposal count (persists across rounds);
+                             * k = out[0] mod n, accepted iff out[1] < P(dE, tau).
+                             * local_flips counts proposals. */
+
 typedef struct abs_config {
     int32_t searches;       /* searches run by this context (per GPU); 0 -> 148 */
     int32_t search_offset;  /* global id of this context's first search
@@ -87,7 +98,13 @@ typedef struct abs_config {
     int32_t trace;          /* async only: 1 = record, per round, the target the
                              * search used and its (B, E_B) (abs_trace_*), so a
                              * run can be replayed exactly; costs host memory */
-    int32_t reserved[7];    /* must be 0 */
+    int32_t policy;         /* ABS_POLICY_WINDOW (default) or ABS_POLICY_SA */
+    int32_t sa_tau_min;     /* SA temperatures ("a different temperature for each */
+    int32_t sa_tau_max;     /* search"): search s (global id) at level     */
+    int32_t sa_levels;      /* j = s mod K has tau = min + (max-min) j / (K-1)
+                             * (integer division); 0 -> min = max(1, max_ij |W_ij|),
+                             * max = min, K = 1 */
+    int32_t reserved[3];    /* must be 0 */
 } abs_config;
 
 typedef struct abs_stats {

@@ -21,6 +21,8 @@ ABS_N_MAX = 32768
 ABS_LADDER_MAX = 32
 MODE_LOCKSTEP = 0
 MODE_ASYNC = 1
+POLICY_WINDOW = 0
+POLICY_SA = 1
 
 
 class AbsError(RuntimeError):
@@ -45,7 +47,11 @@ class abs_config(C.Structure):
         ("external_merge", C.c_int32),
         ("device", C.c_int32),
         ("trace", C.c_int32),
-        ("reserved", C.c_int32 * 7),
+        ("policy", C.c_int32),
+        ("sa_tau_min", C.c_int32),
+        ("sa_tau_max", C.c_int32),
+        ("sa_levels", C.c_int32),
+        ("reserved", C.c_int32 * 3),
     ]
 
 
@@ -164,7 +170,8 @@ def words(n: int) -> int:
 def make_config(n: int, searches: int = 148, search_offset: int = 0, local_flips: int | None = None,
                 pool_size: int = 64, ladder=None, seed: int = 1, p_cross: int = -1, p_mut: int = -1,
                 mut_max: int = 0, mode: int = MODE_LOCKSTEP, external_merge: bool = False,
-                device: int = -1, trace: bool = False) -> abs_config:
+                device: int = -1, trace: bool = False, policy: int = POLICY_WINDOW, sa_tau_min: int = 0,
+                sa_tau_max: int = 0, sa_levels: int = 0) -> abs_config:
     cfg = abs_config()
     load().abs_config_init(C.byref(cfg))
     cfg.searches = int(searches)
@@ -185,6 +192,10 @@ def make_config(n: int, searches: int = 148, search_offset: int = 0, local_flips
     cfg.external_merge = 1 if external_merge else 0
     cfg.device = int(device)
     cfg.trace = 1 if trace else 0
+    cfg.policy = int(policy)
+    cfg.sa_tau_min = int(sa_tau_min)
+    cfg.sa_tau_max = int(sa_tau_max)
+    cfg.sa_levels = int(sa_levels)
     return cfg
 
 

@@ -195,6 +195,8 @@ static void free_ctx(abs_ctx *c)
     cudaFree(c->S.hash);
     cudaFree(c->S.flips);
     cudaFree(c->S.sflips);
+    cudaFree(c->S.tau);
+    cudaFree(c->S.sa_ctr);
     if (c->T_h) cudaFreeHost(c->T_h);
     if (c->B_h) cudaFreeHost(c->B_h);
     if (c->EB_h) cudaFreeHost(c->EB_h);
@@ -263,6 +265,12 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
     if (cfg.mut_max == 0) cfg.mut_max = std::max(1, n / 32);
     if (cfg.mut_max < 0) return fail(ABS_EINVAL, "bad mut_max");
     if (cfg.mode != ABS_MODE_LOCKSTEP && cfg.mode != ABS_MODE_ASYNC) return fail(ABS_EINVAL, "bad mode");
+    if (cfg.policy != ABS_POLICY_WINDOW && cfg.policy != ABS_POLICY_SA) return fail(ABS_EINVAL, "bad policy");
+    if (cfg.sa_tau_min < 0 || cfg.sa_tau_max < 0 || cfg.sa_levels < 0)
+        return fail(ABS_EINVAL, "bad SA temperatures");
+    if (cfg.sa_tau_max != 0 && cfg.sa_tau_max < cfg.sa_tau_min) return fail(ABS_EINVAL, "sa_tau_max < sa_tau_min");
+    for (int i = 0; i < 3; ++i)
+        if (cfg.reserved[i] != 0) return fail(ABS_EINVAL, "reserved config fields must be 0");
     std::vector<int32_t> ladder;
     if (cfg.ladder_len == 0) {
         ladder = default_ladder(n);
@@ -351,6 +359,10 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
         I.wmax = 0;
         for (int32_t v : rm) I.wmax = std::max(I.wmax, v);
     }
+    // SA temperatures (reading E2): defaults from the instance's weight scale
+    if (c->cfg.sa_tau_min == 0) c->cfg.sa_tau_min = std::max(1, I.wmax);
+    if (c->cfg.sa_tau_max == 0) c->cfg.sa_tau_max = c->cfg.sa_tau_min;
+    if (c->cfg.sa_levels == 0) c->cfg.sa_levels = 1;
 
     // ---- per-search state
     SearchState &S = c->S;
@@ -367,6 +379,21 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
     CTX_CU(cudaMalloc(&S.hash, Sn * sizeof(uint64_t)));
     CTX_CU(cudaMalloc(&S.flips, Sn * sizeof(int64_t)));
     CTX_CU(cudaMalloc(&S.sflips, Sn * sizeof(int64_t)));
+    CTX_CU(cudaMalloc(&S.tau, Sn * sizeof(int32_t)));
+    CTX_CU(cudaMalloc(&S.sa_ctr, Sn * sizeof(uint64_t)));
+    CTX_CU(cudaMemsetAsync(S.sa_ctr, 0, Sn * sizeof(uint64_t), c->st));
+    {
+        // search s (global id g) at temperature level j = g mod K (reading E2)
+        const int32_t K = c->cfg.sa_levels, tmin = c->cfg.sa_tau_min, tmax = c->cfg.sa_tau_max;
+        std::vector<int32_t> tv(Sn);
+        for (size_t s = 0; s < Sn; ++s) {
+            const int64_t j = (int64_t)(cfg.search_offset + s) % K;
+            tv[s] = K == 1 ? tmin : (int32_t)(tmin + ((int64_t)(tmax - tmin) * j) / (K - 1));
+        }
+        CTX_CU(cudaMemcpyAsync(S.tau, tv.data(), Sn * sizeof(int32_t), cudaMemcpyHostToDevice, c->st));
+        CTX_CU(cudaStreamSynchronize(c->st));
+        c->h2d += (int64_t)(Sn * sizeof(int32_t));
+    }
     {
         std::vector<int32_t> lv(Sn);
         for (size_t s = 0; s < Sn; ++s) lv[s] = ladder[(size_t)(cfg.search_offset + s) % ladder.size()];
@@ -425,6 +452,11 @@ static int lockstep_step(abs_ctx *c)
     a.sflips = c->S.sflips;
     a.L = c->L;
     a.S = S;
+    a.policy = c->cfg.policy;
+    a.sid0 = c->cfg.search_offset;
+    a.seed = c->cfg.seed;
+    a.tau = c->S.tau;
+    a.sa_ctr = c->S.sa_ctr;
 #ifdef ABS_TIMING
     if (!c->timing_d) {
         ABS_CU(cudaMalloc(&c->timing_d, (size_t)S * 32 * 24 * sizeof(long long)));
@@ -613,6 +645,11 @@ static int async_run(abs_ctx *c, int64_t steps)
     a.sflips = c->S.sflips;
     a.L = c->L;
     a.S = S;
+    a.policy = c->cfg.policy;
+    a.sid0 = c->cfg.search_offset;
+    a.seed = c->cfg.seed;
+    a.tau = c->S.tau;
+    a.sa_ctr = c->S.sa_ctr;
 #ifdef ABS_TIMING
     if (!c->timing_d) {
         ABS_CU(cudaMalloc(&c->timing_d, (size_t)S * 32 * 24 * sizeof(long long)));

@@ -51,6 +51,8 @@ struct SearchState {
     int32_t *a = nullptr, *l = nullptr;
     uint64_t *hash = nullptr;
     int64_t *flips = nullptr, *sflips = nullptr;
+    int32_t *tau = nullptr;         // SA temperature per search
+    uint64_t *sa_ctr = nullptr;     // SA proposals drawn per search (Philox counter)
 };
 
 struct RoundArgs {
@@ -68,6 +70,11 @@ struct RoundArgs {
     int64_t *flips, *sflips;
     int64_t L;
     int32_t S;
+    int32_t policy;          // ABS_POLICY_WINDOW / ABS_POLICY_SA
+    int32_t sid0;            // global id of search 0 (Philox counter word)
+    uint64_t seed;           // Philox key
+    const int32_t *tau;      // SA temperature per search
+    uint64_t *sa_ctr;        // SA proposal counter per search
     long long *timing;  // diagnostics build only: [S][32][8] cycle accumulators
 };
 

@@ -65,6 +65,40 @@ struct MaskOf<64> {
     using T = uint64_t;
 };
 
+constexpr uint32_t kTagSA = 0x5341504Cu;  // 'SAPL'
+
+// Philox4x32-10 (Salmon et al., SC'11), the library's device copy (the oracle
+// has its own; both are pinned by the Random123 known-answer vectors).
+__device__ __forceinline__ void philox4x32_10(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3, uint32_t k0,
+                                              uint32_t k1, uint32_t (&o)[4])
+{
+#pragma unroll
+    for (int r = 0; r < 10; ++r) {
+        const uint32_t hi0 = __umulhi(0xD2511F53u, c0), lo0 = 0xD2511F53u * c0;
+        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c2), lo1 = 0xCD9E8D57u * c2;
+        c0 = hi1 ^ c1 ^ k0;
+        c1 = lo1;
+        c2 = hi0 ^ c3 ^ k1;
+        c3 = lo0;
+        k0 += 0x9E3779B9u;
+        k1 += 0xBB67AE85u;
+    }
+    o[0] = c0;
+    o[1] = c1;
+    o[2] = c2;
+    o[3] = c3;
+}
+
+// SA acceptance bound of an uphill move (reading E2): Eq.(7) as 2^(-dE/tau),
+// linear between integer exponents, in Q32: accept iff a uniform uint32 < it.
+__device__ __forceinline__ uint64_t sa_threshold(int dE, int tau)
+{
+    const int q = dE / tau;
+    const int rem = dE - q * tau;
+    if (q >= 32) return 0;
+    return ((uint64_t)1 << (32 - q)) * (uint64_t)(2 * (long long)tau - rem) / (uint64_t)(2 * (long long)tau);
+}
+
 struct Red {
     int v;  // min Delta over all bits (neighbour tracking)
     int c;  // min Delta over the candidate set
@@ -80,6 +114,9 @@ struct RoundSmem {
     long long E, EB, LB;  // E(X), E_B, lower bound on min_i Delta_i(X): thread 0 only
     unsigned long long hash;
     long long nflip, nstraight;
+    unsigned long long sa_ctr;  // SA: proposals drawn (Philox counter); thread 0 writes
+    int sa_tau;                 // SA: this search's temperature
+    int sa_d[2], sa_x[2];       // SA: Delta_k / x_k of the proposal, by counter parity
 #ifdef ABS_TIMING
     long long tacc[32][24];  // [warp][local 0-6 | straight 8-14 | selection sub-phases 16-20]
 #endif
@@ -89,7 +126,7 @@ struct WindowSmem {  // published Delta / x of the next window, by flip parity
     uint8_t x[2][kWinMax];
 };
 
-template <int kP, int kMaxT, int kNT>
+template <int kP, int kMaxT, int kNT, bool kSA>
 struct Round {
     static constexpr int G = kP / 8;  // byte-groups per thread
     static constexpr bool kMulti = kMaxT > 32;
@@ -355,6 +392,51 @@ struct Round {
         }
     }
 
+    // SA policy (Alg. 1 + Eq.(7), reading E2): draw proposals until one is
+    // accepted or the round's proposal budget `left` is spent.  The owner of
+    // bit k broadcasts Delta_k and x_k through shared memory (slot = counter
+    // parity, one barrier per proposal).  Returns false when nothing was accepted.
+    static __device__ __forceinline__ bool sa_next(const RoundArgs &A, RoundSmem *sm, const int (&g)[kP], M xm,
+                                                   int sid, int n, int t, int nt, int &left, int &k, int &dk, int &xk)
+    {
+        unsigned long long c = sm->sa_ctr;  // written by thread 0 before the last barrier
+        const int tau = sm->sa_tau;
+        const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
+        bool acc = false;
+        while (left > 0) {
+            --left;
+            uint32_t o[4];
+            philox4x32_10((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
+            const int par = (int)(c & 1u);
+            ++c;
+            const int kk = (int)(o[0] % (uint32_t)n);  // "randomly select a bit" (Alg. 1)
+            const int j = group_of(kk, nt);
+            if (t == (kk >> 3) - nt * j) {
+                const int e = kk & 7;
+                int v = 0;
+#pragma unroll
+                for (int jj = 0; jj < G; ++jj)
+#pragma unroll
+                    for (int ee = 0; ee < 8; ++ee)
+                        if (jj == j && ee == e) v = g[8 * jj + ee];
+                sm->sa_d[par] = readout(v, xm, 8 * j + e);
+                sm->sa_x[par] = (int)bit(xm, 8 * j + e);
+            }
+            sync();
+            const int d = sm->sa_d[par];
+            const int x = sm->sa_x[par];
+            if (d <= 0 || (uint64_t)o[1] < sa_threshold(d, tau)) {  // Eq.(7)
+                k = kk;
+                dk = d;
+                xk = x;
+                acc = true;
+                break;
+            }
+        }
+        if (t == 0) sm->sa_ctr = c;
+        return acc;
+    }
+
     static __device__ __forceinline__ void init_barriers(unsigned char *smem)
     {
         RoundSmem *sm = reinterpret_cast<RoundSmem *>(smem);
@@ -402,6 +484,8 @@ struct Round {
             sm->E = A.E[sid];
             sm->EB = sm->E;  // Step 3, reading C4: E_B = E(C) (Alg. 5) ...
             sm->LB = INT64_MIN / 4;
+            sm->sa_ctr = A.policy == 1 ? A.sa_ctr[sid] : 0ull;
+            sm->sa_tau = A.policy == 1 ? A.tau[sid] : 1;
         }
 
         // ---- the search state (registers for the whole round)
@@ -425,15 +509,19 @@ struct Round {
         }
         int a = A.a[sid];
         const int l = A.l[sid];
-        const bool pre = kMulti && l <= kWinMax;
+        constexpr bool sa = kSA;  // ABS_POLICY_SA: a separate kernel instantiation
+        const bool pre = kMulti && l <= kWinMax && !sa;
         int left = (int)A.L;
         int rb = 0;
         sync();
 
         // ---- first selection of the round
         bool straight = block_any(xm != stm[t]);
-        int k, dk, xk;
-        {
+        int k = 0, dk = 0, xk = 0;
+        bool have = true;  // a first flip exists (SA may accept nothing)
+        if (sa && !straight) {
+            have = sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk);
+        } else {
             int cv, ci2;
             if constexpr (kMulti) {  // one inlined scan (code size of the flip loop)
                 const M cm = straight ? (M)(xm ^ stm[t]) : window_mask(a, l, n, t, nt);
@@ -453,11 +541,11 @@ struct Round {
             dk = r.c;
         }
         bool exact = true;  // compute the n neighbour deltas of this flip exactly
-        if (t == ctl) issue_row(A, k, rowbuf + rowb * (fbase & 1), sm->bar[fbase & 1], nt);
+        if (have && t == ctl) issue_row(A, k, rowbuf + rowb * (fbase & 1), sm->bar[fbase & 1], nt);
 
         int f = 0;
         ABS_T(if (lane == 0) for (int q = 0; q < 24; ++q) sm->tacc[warp][q] = 0;)
-        for (;; ++f) {
+        for (; have; ++f) {
             const int b = (fbase + f) & 1;
             const uint32_t par = (uint32_t)((fbase + f) >> 1) & 1u;
             unsigned char *row = rowbuf + rowb * b;
@@ -555,8 +643,10 @@ struct Round {
             } else {
                 if (exact) process_row<kMin>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
                 else process_row<kUpdate>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
-                a += l;  // offset <- (a + l) mod n
-                if (a >= n) a -= n;
+                if (!sa) {
+                    a += l;  // offset <- (a + l) mod n
+                    if (a >= n) a -= n;
+                }
             }
             ABS_T(long long tc3 = clock64();)
             int ci2 = INT_MAX;
@@ -565,7 +655,7 @@ struct Round {
                     int a2 = a + l;
                     if (a2 >= n) a2 -= n;
                     publish_window(g, xm, a2, l, n, t, nt, win->d[b ^ 1], win->x[b ^ 1]);
-                } else {
+                } else if (!sa) {
                     window_candidates(g, xm, a, l, n, t, nt, cmin, ci2);
                 }
             }
@@ -632,7 +722,15 @@ struct Round {
             }
 
             // ---- next flip
-            if (!straight) {
+            if (!straight && sa) {
+                if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk)) break;
+                if constexpr (!kMulti) {
+                    __syncwarp();
+                    const long long E1 = sm->E;
+                    const long long LB2 = min(sm->LB - 2 * (long long)A.wmax, -(long long)dk);
+                    exact = E1 + dk + min(LB2, 0LL) < sm->EB;
+                }
+            } else if (!straight) {
                 if (--left <= 0) break;
                 if (pre) {
                     const int4 sv = sm->sel[b];
@@ -667,6 +765,12 @@ struct Round {
                 // X = T: the straight search is over; local search from T (Step 4b)
                 straight = false;
                 if (left <= 0) break;
+                if (sa) {
+                    if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk)) break;
+                    exact = true;
+                    if (t == ctl) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+                    continue;
+                }
                 int cv, cj;
                 if constexpr (kMulti) candidates(g, xm, window_mask(a, l, n, t, nt), t, nt, cv, cj);
                 else candidates_window(g, xm, a, l, n, t, nt, cv, cj);
@@ -694,7 +798,7 @@ struct Round {
             })
         }
 
-        fbase += f + 1;  // rows consumed in this round (no row left in flight)
+        if (have) fbase += f + 1;  // rows consumed in this round (no row left in flight)
         ABS_T(if (lane == 0 && A.timing) for (int q = 0; q < 24; ++q)
                   atomicAdd((unsigned long long *)&A.timing[((size_t)sid * 32 + warp) * 24 + q],
                             (unsigned long long)sm->tacc[warp][q]);)
@@ -722,23 +826,24 @@ struct Round {
                 A.a[sid] = a;
                 A.hash[sid] = sm->hash;
                 A.flips[sid] += sm->nflip;
+                if (sa) A.sa_ctr[sid] = sm->sa_ctr;
                 A.sflips[sid] += sm->nstraight;
             }
         }
     }
 };
 
-template <int kP, int kMaxT, int kNT>
+template <int kP, int kMaxT, int kNT, bool kSA>
 __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (kMaxT == 128 ? 6 : 1)) round_kernel(const RoundArgs A)
 {
     extern __shared__ __align__(128) unsigned char smem[];
     const int sid = blockIdx.x;
     const size_t bpv = (size_t)A.n_pad / 8;
     int fbase = 0;
-    Round<kP, kMaxT, kNT>::init_barriers(smem);
+    Round<kP, kMaxT, kNT, kSA>::init_barriers(smem);
     uint8_t *const B0 = A.B + sid * bpv;
     int64_t *const EB0 = A.EB + sid;
-    Round<kP, kMaxT, kNT>::run(
+    Round<kP, kMaxT, kNT, kSA>::run(
         A, smem, sid, A.T + sid * bpv,
         [=](uint8_t *&Bp, int64_t *&EBp) {
             Bp = B0;
@@ -779,7 +884,7 @@ __device__ __forceinline__ void st_release_gpu(int *p, int v)
 // system-scope release and appends (search, round) to an arrival ring the host
 // GA polls.
 // Host and device never synchronise directly.
-template <int kP, int kMaxT, int kNT>
+template <int kP, int kMaxT, int kNT, bool kSA>
 __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (kMaxT == 128 ? 6 : 1))
     round_kernel_async(const RoundArgs A, const AsyncArgs Q)
 {
@@ -792,7 +897,7 @@ __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (k
     const size_t bpv = (size_t)A.n_pad / 8;
     constexpr bool multi = kMaxT > 32;
     int fbase = 0;
-    Round<kP, kMaxT, kNT>::init_barriers(smem);
+    Round<kP, kMaxT, kNT, kSA>::init_barriers(smem);
     if (threadIdx.x == 0) r_own = Q.owned ? ld_acquire_gpu(Q.done + blockIdx.x) : 0;
     for (;;) {
         if (threadIdx.x == 0) {
@@ -823,7 +928,7 @@ __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (k
         if (multi) __syncthreads();
         else __syncwarp();
         if (item >= Q.total) break;
-        Round<kP, kMaxT, kNT>::run(
+        Round<kP, kMaxT, kNT, kSA>::run(
             A, smem, cur_s, Q.Tmap + ((size_t)cur_s * 2 + (tver & 1)) * bpv,
             [&](uint8_t *&Bp, int64_t *&EBp) {
                 const int s = cur_s, r = cur_r;
@@ -852,16 +957,16 @@ __global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (k
     }
 }
 
-template <int kP, int kMaxT, int kNT>
-int launch_variant(const RoundArgs &a, cudaStream_t st, size_t smem, const AsyncArgs *q, int *grid_out)
+template <int kP, int kMaxT, int kNT, bool kSA>
+int launch_policy(const RoundArgs &a, cudaStream_t st, size_t smem, const AsyncArgs *q, int *grid_out)
 {
     if (!q) {
-        auto k = round_kernel<kP, kMaxT, kNT>;
+        auto k = round_kernel<kP, kMaxT, kNT, kSA>;
         cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
         k<<<a.S, a.nt, smem, st>>>(a);
         return (int)cudaGetLastError();
     }
-    auto k = round_kernel_async<kP, kMaxT, kNT>;
+    auto k = round_kernel_async<kP, kMaxT, kNT, kSA>;
     cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     int per_sm = 0, dev = 0, sms = 0;
     cudaGetDevice(&dev);
@@ -887,9 +992,16 @@ size_t round_smem_bytes(int32_t nt, int32_t bpt)
 }
 
 template <int kP, int kMaxT, int kNT>
+int launch_variant(const RoundArgs &a, cudaStream_t st, size_t smem, const AsyncArgs *q, int *grid_out)
+{
+    if (a.policy == 1) return launch_policy<kP, kMaxT, kNT, true>(a, st, smem, q, grid_out);
+    return launch_policy<kP, kMaxT, kNT, false>(a, st, smem, q, grid_out);
+}
+
+template <int kP, int kMaxT, int kNT>
 int occupancy_variant(int nt, size_t smem, int *per_sm)
 {
-    auto k = round_kernel<kP, kMaxT, kNT>;
+    auto k = round_kernel<kP, kMaxT, kNT, false>;
     cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     return (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k, nt, smem);
 }
