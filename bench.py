@@ -224,6 +224,10 @@ def run_abs(args):
     Wd = Wp.to(f"cuda:{local}", non_blocking=False)
     mode = pkg.MODE_ASYNC if args.mode == "async" else pkg.MODE_LOCKSTEP
     common = dict(searches=S, local_flips=L, pool_size=64, seed=1, device=local, mode=mode)
+    if args.policy == "sa":
+        # SA policy (reading E2): a 4-level temperature ladder from the weight scale up
+        wmax = int(np.abs(W[:256].astype(np.int32)).max()) or 1  # weight scale from a row sample
+        common.update(policy=pkg.POLICY_SA, sa_tau_min=max(1, wmax // 4), sa_tau_max=8 * wmax, sa_levels=4)
     solver = pkg.Solver(Wd, search_offset=rank * S, external_merge=(world > 1 and mode == pkg.MODE_LOCKSTEP),
                         **common)
     del Wd
@@ -360,7 +364,7 @@ def run_abs(args):
             "data": "synthetic (Philox random int16 QUBO, P:L468)" if args.workload.startswith("random")
             else "synthetic",
             "config": {"workload": args.workload, "desc": WORKLOADS[args.workload], "n": n,
-                       "searches_per_gpu": S, "local_flips": L, "pool": 64, "mode": args.mode,
+                       "searches_per_gpu": S, "local_flips": L, "pool": 64, "mode": args.mode, "policy": args.policy,
                        "parallelism": "dp%d (replicated W, independent searches)" % world,
                        "l2": "inputs larger than L2 (W = %d MiB)" % (2 * n * n >> 20)
                        if 2 * n * n > 126 * 2 ** 20 else "W fits in L2 (resident by design)"},
@@ -387,6 +391,7 @@ def main():
     ap.add_argument("--workload", default="random32k", choices=sorted(WORKLOADS))
     ap.add_argument("--searches", type=int, default=0)
     ap.add_argument("--mode", default="lockstep", choices=["lockstep", "async"])
+    ap.add_argument("--policy", default="window", choices=["window", "sa"])
     ap.add_argument("--local-flips", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
