@@ -126,6 +126,9 @@ typedef struct abs_stats {
                                * from entry to exit of every abs_search call,
                                * host GA gaps included */
     int64_t round_kernel_launches; /* launches of the search (round) kernel */
+    double init_seconds;      /* device time of the last batched initialisation
+                               * (abs_energy / abs_energy_dev / abs_seed_pool;
+                               * CUDA events around its kernels) */
 } abs_stats;
 
 typedef struct abs_ctx abs_ctx;
@@ -186,6 +189,25 @@ ABS_API int abs_pool_insert(abs_ctx *c, const uint32_t *X, const int64_t *E, int
  * E (Eq.(1)) and, if delta_out != NULL, all Delta_i (Eq.(13)) on the
  * device.  E_out: count int64; delta_out: count*n int32 (row-major). */
 ABS_API int abs_energy(abs_ctx *c, const uint32_t *X, int32_t count, int64_t *E_out, int32_t *delta_out);
+
+/* Engines of the batched initialisation. */
+#define ABS_INIT_AUTO 0 /* the tensor-core engine */
+#define ABS_INIT_ALU 1  /* plain integer kernel: conditional row adds, W read once per 16 solutions */
+#define ABS_INIT_MMA 2  /* tensor cores: S = X Wz^T as two exact int8 GEMMs,
+                         * W = 256 hi + lo (hi s8, lo u8), tcgen05.mma kind::i8 with int32
+                         * TMEM accumulators; the int8 planes of W (2 n_pad^2 bytes) are
+                         * built on first use and kept with the context */
+
+/* Batched initialisation on DEVICE buffers (same operation as abs_energy,
+ * Eq.(1) and Eq.(13)): X_dev = count bit vectors of
+ * words(n) uint32 each (ABI bit order; bits >= n ignored), E_dev = count
+ * int64 (overwritten), delta_dev = count*n int32 row-major or NULL.  All
+ * pointers are device memory of the context's device, owned by the caller.
+ * Blocking; results are exact in every engine.  ABS_EINVAL for bad
+ * arguments or engine, ABS_ENOMEM if the planes / staging cannot be
+ * allocated, ABS_ECUDA on a CUDA error. */
+ABS_API int abs_energy_dev(abs_ctx *c, const uint32_t *X_dev, int32_t count, int64_t *E_dev, int32_t *delta_dev,
+                           int32_t engine);
 
 /* Lockstep: the (B, E_B) every local search emitted in the last step, in
  * local search order.  B_out: searches*words(n) words, EB_out: searches. */

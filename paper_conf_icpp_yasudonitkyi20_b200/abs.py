@@ -73,12 +73,13 @@ class abs_stats(C.Structure):
         ("kernel_launches", C.c_int64),
         ("step_seconds", C.c_double),
         ("round_kernel_launches", C.c_int64),
+        ("init_seconds", C.c_double),
     ]
 
 
 EXPORTS = [
     "abs_config_init", "abs_create", "abs_create_dev", "abs_seed_pool", "abs_search", "abs_best",
-    "abs_stats_get", "abs_pool_get", "abs_pool_insert", "abs_energy", "abs_round_results",
+    "abs_stats_get", "abs_pool_get", "abs_pool_insert", "abs_energy", "abs_energy_dev", "abs_round_results",
     "abs_round_targets", "abs_trace_count", "abs_trace_get", "abs_search_state", "abs_debug_timing", "abs_destroy", "abs_strerror", "abs_last_error", "abs_device_searches", "abs_ising_to_qubo", "abs_qubo_to_ising", "abs_version",
 ]
 
@@ -117,6 +118,8 @@ def load(build_if_missing: bool = True):
     L.abs_pool_get.argtypes = [vp, C.c_int32, vp, vp, P(C.c_int32)]
     L.abs_pool_insert.argtypes = [vp, vp, vp, C.c_int32, P(C.c_int32)]
     L.abs_energy.argtypes = [vp, vp, C.c_int32, vp, vp]
+    if hasattr(L, "abs_energy_dev") or not os.environ.get("ABS_LIB"):
+        L.abs_energy_dev.argtypes = [vp, vp, C.c_int32, vp, vp, C.c_int32]
     L.abs_round_results.argtypes = [vp, vp, vp]
     L.abs_round_targets.argtypes = [vp, vp]
     L.abs_trace_count.argtypes = [vp, P(C.c_int64)]
@@ -161,6 +164,9 @@ def _check(rc: int, where: str):
 
 def _ptr(a):
     return None if a is None else C.c_void_p(a.ctypes.data)
+
+
+INIT_AUTO, INIT_ALU, INIT_MMA = 0, 1, 2  # batched-init engines (include/abs.h)
 
 
 def words(n: int) -> int:
@@ -291,6 +297,21 @@ class Solver:
         D = np.zeros((cnt, self.n), np.int32) if want_delta else None
         _check(load().abs_energy(self._c, _ptr(X), cnt, _ptr(E), _ptr(D)), "abs_energy")
         return (E, D) if want_delta else E
+
+    def energy_dev(self, X, E, D=None, engine: int = INIT_AUTO) -> float:
+        """abs_energy_dev on CUDA torch tensors: X int32/uint32-bit words
+        [count, words], E int64 [count] (written), D int32 [count, n] or None.
+        Returns the device time of the launch (seconds, CUDA events)."""
+        import torch
+        assert X.is_cuda and X.dtype == torch.int32 and X.shape[1] == self.words and X.is_contiguous()
+        cnt = int(X.shape[0])
+        assert E.is_cuda and E.dtype == torch.int64 and E.numel() >= cnt
+        if D is not None:
+            assert D.is_cuda and D.dtype == torch.int32 and D.is_contiguous() and D.numel() >= cnt * self.n
+        torch.cuda.synchronize(X.device)
+        _check(load().abs_energy_dev(self._c, C.c_void_p(X.data_ptr()), cnt, C.c_void_p(E.data_ptr()),
+                                     None if D is None else C.c_void_p(D.data_ptr()), int(engine)), "abs_energy_dev")
+        return float(self.stats()["init_seconds"])
 
     def round_results(self):
         B = np.zeros((self.searches, self.words), np.uint32)

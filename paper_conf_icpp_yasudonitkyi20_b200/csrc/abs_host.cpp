@@ -174,6 +174,12 @@ struct abs_ctx {
     std::vector<TraceEntry> trace;
     int async_grid = 0;
     long long *timing_d = nullptr;  // diagnostics build
+    // ---- tensor-core batched init: W int8 planes (built on first use), A staging
+    int8_t *Whi = nullptr;
+    uint8_t *Wlo = nullptr;
+    uint8_t *Ainit = nullptr;
+    size_t Ainit_bytes = 0;
+    double init_ms = 0.0;  // last batched-init launch (CUDA events)
 };
 
 static void free_ctx(abs_ctx *c)
@@ -184,6 +190,9 @@ static void free_ctx(abs_ctx *c)
     cudaFree(c->I.Wz);
     cudaFree(c->I.diag);
     cudaFree(c->I.rowmax);
+    cudaFree(c->Whi);
+    cudaFree(c->Wlo);
+    cudaFree(c->Ainit);
     cudaFree(c->S.g);
     cudaFree(c->S.X);
     cudaFree(c->S.B);
@@ -728,45 +737,94 @@ int abs_create_dev(abs_ctx **out, int32_t n, const int16_t *W_dev, const abs_con
     }
 }
 
+// Batched init on device buffers: X_dev packed words, row
+// stride words(n); E_dev count int64; delta_dev count*n int32 or NULL.
+static int energy_device(abs_ctx *c, const uint32_t *X_dev, int32_t count, int64_t *E_dev, int32_t *delta_dev,
+                         int32_t engine)
+{
+    const int row_bytes = 4 * words_of(c->I.n);
+    const uint8_t *X = reinterpret_cast<const uint8_t *>(X_dev);
+    if (engine == ABS_INIT_ALU) {
+        ABS_CU(cudaEventRecord(c->ev0, c->st));
+        ABS_CK(launch_batch_init(c->I, X, row_bytes, count, E_dev, delta_dev, c->st));
+        ABS_CU(cudaEventRecord(c->ev1, c->st));
+        c->launches += 1;
+    } else {
+        if (!c->Whi) {  // int8 planes of W, once per instance
+            const size_t pb = init_mma_plane_bytes(c->I.n_pad);
+            if (cudaMalloc(&c->Whi, pb) != cudaSuccess) return fail(ABS_ENOMEM, "W hi plane");
+            if (cudaMalloc(&c->Wlo, pb) != cudaSuccess) return fail(ABS_ENOMEM, "W lo plane");
+            ABS_CK(launch_wsplit(c->I, c->Whi, c->Wlo, c->st));
+            c->launches += 1;
+        }
+        const size_t ab = init_mma_a_bytes(count, c->I.n_pad);
+        if (ab > c->Ainit_bytes) {
+            cudaFree(c->Ainit);
+            c->Ainit = nullptr;
+            c->Ainit_bytes = 0;
+            if (cudaMalloc(&c->Ainit, ab) != cudaSuccess) return fail(ABS_ENOMEM, "init A staging");
+            c->Ainit_bytes = ab;
+        }
+        ABS_CU(cudaEventRecord(c->ev0, c->st));
+        ABS_CK(launch_init_mma(c->I, c->Whi, c->Wlo, X, row_bytes, count, c->Ainit, E_dev, delta_dev, c->st));
+        ABS_CU(cudaEventRecord(c->ev1, c->st));
+        c->launches += 2;
+    }
+    return ABS_OK;
+}
+
+int abs_energy_dev(abs_ctx *c, const uint32_t *X_dev, int32_t count, int64_t *E_dev, int32_t *delta_dev,
+                   int32_t engine)
+{
+    if (!c || count < 0 || (count > 0 && (!X_dev || !E_dev))) return fail(ABS_EINVAL, "bad arguments");
+    if (engine != ABS_INIT_AUTO && engine != ABS_INIT_ALU && engine != ABS_INIT_MMA)
+        return fail(ABS_EINVAL, "unknown engine");
+    if (count == 0) return ABS_OK;
+    ABS_CU(cudaSetDevice(c->device));
+    const int rc = energy_device(c, X_dev, count, E_dev, delta_dev, engine);
+    if (rc) return rc;
+    ABS_CU(cudaStreamSynchronize(c->st));
+    float ms = 0.f;
+    ABS_CU(cudaEventElapsedTime(&ms, c->ev0, c->ev1));
+    c->init_ms = ms;
+    return ABS_OK;
+}
+
 int abs_energy(abs_ctx *c, const uint32_t *X, int32_t count, int64_t *E_out, int32_t *delta_out)
 {
     if (!c || (count > 0 && (!X || !E_out)) || count < 0) return fail(ABS_EINVAL, "bad arguments");
     if (count == 0) return ABS_OK;
-    try {
-        ABS_CU(cudaSetDevice(c->device));
-        const int n = c->I.n, words = words_of(n), bpv = c->bytes_per_vec;
-        std::vector<uint8_t> xb((size_t)count * bpv);
-        for (int b = 0; b < count; ++b) words_to_bytes(X + (size_t)b * words, words, &xb[(size_t)b * bpv], bpv, n);
-        uint8_t *X_d = nullptr;
-        int64_t *E_d = nullptr;
-        int32_t *D_d = nullptr;
-        auto cleanup = [&]() {
-            cudaFree(X_d);
-            cudaFree(E_d);
-            cudaFree(D_d);
-        };
-        cudaError_t e = cudaMalloc(&X_d, xb.size());
-        if (e == cudaSuccess) e = cudaMalloc(&E_d, sizeof(int64_t) * (size_t)count);
-        if (e == cudaSuccess && delta_out) e = cudaMalloc(&D_d, sizeof(int32_t) * (size_t)count * n);
-        if (e == cudaSuccess) e = cudaMemcpyAsync(X_d, xb.data(), xb.size(), cudaMemcpyHostToDevice, c->st);
-        if (e == cudaSuccess) {
-            const int rc = launch_batch_init(c->I, X_d, count, E_d, D_d, c->st);
-            c->launches++;
-            e = (cudaError_t)rc;
-        }
-        if (e == cudaSuccess)
-            e = cudaMemcpyAsync(E_out, E_d, sizeof(int64_t) * (size_t)count, cudaMemcpyDeviceToHost, c->st);
+    ABS_CU(cudaSetDevice(c->device));
+    const int n = c->I.n, words = words_of(n);
+    uint32_t *X_d = nullptr;
+    int64_t *E_d = nullptr;
+    int32_t *D_d = nullptr;
+    auto cleanup = [&]() {
+        cudaFree(X_d);
+        cudaFree(E_d);
+        cudaFree(D_d);
+    };
+    const size_t xbytes = sizeof(uint32_t) * (size_t)count * words;
+    cudaError_t e = cudaMalloc(&X_d, xbytes);
+    if (e == cudaSuccess) e = cudaMalloc(&E_d, sizeof(int64_t) * (size_t)count);
+    if (e == cudaSuccess && delta_out) e = cudaMalloc(&D_d, sizeof(int32_t) * (size_t)count * n);
+    if (e != cudaSuccess) {
+        cleanup();
+        return fail(ABS_ENOMEM, std::string("abs_energy: ") + cudaGetErrorString(e));
+    }
+    e = cudaMemcpyAsync(X_d, X, xbytes, cudaMemcpyHostToDevice, c->st);
+    int rc = (e == cudaSuccess) ? energy_device(c, X_d, count, E_d, D_d, ABS_INIT_AUTO) : ABS_ECUDA;
+    if (rc == ABS_OK) {
+        e = cudaMemcpyAsync(E_out, E_d, sizeof(int64_t) * (size_t)count, cudaMemcpyDeviceToHost, c->st);
         if (e == cudaSuccess && delta_out)
             e = cudaMemcpyAsync(delta_out, D_d, sizeof(int32_t) * (size_t)count * n, cudaMemcpyDeviceToHost, c->st);
         if (e == cudaSuccess) e = cudaStreamSynchronize(c->st);
-        cleanup();
-        c->h2d += (int64_t)xb.size();
-        c->d2h += (int64_t)count * 8 + (delta_out ? (int64_t)count * n * 4 : 0);
-        if (e != cudaSuccess) return fail(ABS_ECUDA, std::string("abs_energy: ") + cudaGetErrorString(e));
-        return ABS_OK;
-    } catch (const std::bad_alloc &) {
-        return fail(ABS_ENOMEM, "host allocation");
+        if (e != cudaSuccess) rc = fail(ABS_ECUDA, std::string("abs_energy: ") + cudaGetErrorString(e));
     }
+    cleanup();
+    c->h2d += (int64_t)xbytes;
+    c->d2h += (int64_t)count * 8 + (delta_out ? (int64_t)count * n * 4 : 0);
+    return rc;
 }
 
 int abs_seed_pool(abs_ctx *c, const uint32_t *X, int32_t count)
@@ -856,6 +914,7 @@ int abs_stats_get(const abs_ctx *c, abs_stats *s)
     s->kernel_launches = c->launches;
     s->step_seconds = c->step_seconds;
     s->round_kernel_launches = c->round_launches;
+    s->init_seconds = c->init_ms * 1e-3;
     return ABS_OK;
 }
 

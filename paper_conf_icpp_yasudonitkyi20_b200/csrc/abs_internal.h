@@ -106,10 +106,19 @@ int launch_zero_start(const Instance &I, SearchState &S, int32_t s0, int32_t s1,
 // q == nullptr: lockstep round (one CTA per search); otherwise the persistent
 // asynchronous kernel (grid = min(S, resident CTAs), *grid_out).
 int launch_round(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q = nullptr, int *grid_out = nullptr);
-// Batched init: X bytes [count][n_pad/8] -> E [count], and either
+// Batched init, ALU kernel: X packed bits, row b at X + b * row_bytes
+// (row_bytes a multiple of 4; bits >= n ignored) -> E [count], and either
 // Delta int32 [count][n] (plain layout) or nothing.
-int launch_batch_init(const Instance &I, const uint8_t *X, int32_t count, int64_t *E, int32_t *delta,
-                      cudaStream_t st);
+int launch_batch_init(const Instance &I, const uint8_t *X, int32_t row_bytes, int32_t count, int64_t *E,
+                      int32_t *delta, cudaStream_t st);
+// Batched init on the tensor cores (abs_init_mma.cu): W split once
+// into int8 planes hi / lo (n_pad * n_pad bytes each, UMMA block layout), X
+// expanded per call into A (init_mma_a_bytes), then tcgen05.mma kind::i8.
+size_t init_mma_plane_bytes(int32_t n_pad);
+size_t init_mma_a_bytes(int32_t count, int32_t n_pad);
+int launch_wsplit(const Instance &I, int8_t *hi, uint8_t *lo, cudaStream_t st);
+int launch_init_mma(const Instance &I, const int8_t *hi, const uint8_t *lo, const uint8_t *X, int32_t row_bytes,
+                    int32_t count, uint8_t *A, int64_t *E, int32_t *delta, cudaStream_t st);
 size_t round_smem_bytes(int32_t nt, int32_t bpt);
 // CTAs of the round kernel for layout (nt, bpt) resident per SM (cudaError_t).
 int round_occupancy(int32_t nt, int32_t bpt, int *per_sm);

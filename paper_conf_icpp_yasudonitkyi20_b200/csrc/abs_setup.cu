@@ -98,8 +98,9 @@ constexpr int kInitB = 16;
 constexpr int kInitT = 256;
 __global__ void __launch_bounds__(kInitT) batch_init_kernel(const int16_t *__restrict__ Wz,
                                                             const int32_t *__restrict__ diag, int n, int n_pad,
-                                                            const uint8_t *__restrict__ X, int count,
-                                                            int64_t *__restrict__ Eout, int32_t *__restrict__ delta)
+                                                            const uint8_t *__restrict__ X, int row_bytes,
+                                                            int count, int64_t *__restrict__ Eout,
+                                                            int32_t *__restrict__ delta)
 {
     extern __shared__ uint32_t sx[];  // [kInitB][n_pad/32]
     __shared__ long long red[kInitB][kInitT / 32];
@@ -109,9 +110,10 @@ __global__ void __launch_bounds__(kInitT) batch_init_kernel(const int16_t *__res
     for (int q = threadIdx.x; q < kInitB * words; q += kInitT) {
         const int b = q / words, w = q % words;
         uint32_t v = 0;
-        if (b0 + b < count) {
-            const uint8_t *xb = X + (size_t)(b0 + b) * (n_pad / 8) + 4 * w;
+        if (b0 + b < count && 32 * w < n && 4 * w < row_bytes) {  // row_bytes: a multiple of 4
+            const uint8_t *xb = X + (size_t)(b0 + b) * row_bytes + 4 * w;
             v = (uint32_t)xb[0] | ((uint32_t)xb[1] << 8) | ((uint32_t)xb[2] << 16) | ((uint32_t)xb[3] << 24);
+            if (n - 32 * w < 32) v &= (1u << (n - 32 * w)) - 1u;  // bits >= n are ignored
         }
         sx[b * words + w] = v;
     }
@@ -181,15 +183,15 @@ int launch_zero_start(const Instance &I, SearchState &S, int32_t s0, int32_t s1,
     return (int)cudaGetLastError();
 }
 
-int launch_batch_init(const Instance &I, const uint8_t *X, int32_t count, int64_t *E, int32_t *delta,
-                      cudaStream_t st)
+int launch_batch_init(const Instance &I, const uint8_t *X, int32_t row_bytes, int32_t count, int64_t *E,
+                      int32_t *delta, cudaStream_t st)
 {
     if (count <= 0) return 0;
     cudaMemsetAsync(E, 0, sizeof(int64_t) * (size_t)count, st);
     dim3 grid(I.n_pad / kInitT, (count + kInitB - 1) / kInitB);
     const size_t smem = (size_t)kInitB * (I.n_pad / 32) * sizeof(uint32_t);
     cudaFuncSetAttribute(batch_init_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    batch_init_kernel<<<grid, kInitT, smem, st>>>(I.Wz, I.diag, I.n, I.n_pad, X, count, E, delta);
+    batch_init_kernel<<<grid, kInitT, smem, st>>>(I.Wz, I.diag, I.n, I.n_pad, X, row_bytes, count, E, delta);
     return (int)cudaGetLastError();
 }
 
