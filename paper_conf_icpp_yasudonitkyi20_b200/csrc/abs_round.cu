@@ -309,12 +309,15 @@ struct Round {
     // min over all bits (vmin) and, kMode == kStraight, over the mismatches (cmin).
     template <int kMode>
     static __device__ __forceinline__ void process_row(int (&g)[kP], M xm, M mism, const uint4 *row4, uint64_t *bars,
-                                                       uint32_t par, int c, int t, int nt, int &vmin, int &cmin)
+                                                       uint32_t par, int c, int t, int nt, int &vmin, int &cmin,
+                                                       int &cj)
     {
         vmin = INT_MAX;
         cmin = INT_MAX;
+        cj = 0;  // kStraight: first byte-group holding cmin (lowest index, reading C5)
 #pragma unroll
         for (int j = 0; j < G; ++j) {
+            int gmin = INT_MAX;
             if (kRowChunks == 2 ? (j % (G / 2) == 0) : (j == 0)) mbar_wait(&bars[kRowChunks == 2 ? j / (G / 2) : 0], par);
             const uint4 w4 = row4[t + nt * j];
             const uint32_t wv[4] = {w4.x, w4.y, w4.z, w4.w};
@@ -330,11 +333,34 @@ struct Round {
                     if (kMode == kStraight) {
                         const int m0 = bit(mism, s0) ? d0 : INT_MAX;
                         const int m1 = bit(mism, s0 + 1) ? d1 : INT_MAX;
-                        cmin = min(cmin, min(m0, m1));
+                        gmin = min(gmin, min(m0, m1));
                     }
                 }
             }
+            if (kMode == kStraight && gmin < cmin) {
+                cmin = gmin;
+                cj = j;
+            }
         }
+    }
+
+    // 2*index + x of the lowest mismatch slot of byte-group jsel whose Delta
+    // equals v (INT_MAX if none): the straight phase's argmin index (Alg. 5),
+    // scanning 8 slots instead of P.
+    static __device__ __forceinline__ int lowest_equal_group(const int (&g)[kP], M xm, M cm, int v, int jsel, int t,
+                                                             int nt)
+    {
+        int r = INT_MAX;
+#pragma unroll
+        for (int j = 0; j < G; ++j) {
+            if (j != jsel) continue;
+#pragma unroll
+            for (int e = 7; e >= 0; --e) {
+                const int s = 8 * j + e;
+                if (bit(cm, s) && readout(g[s], xm, s) == v) r = 2 * slot_index(t, nt, s) + (int)bit(xm, s);
+            }
+        }
+        return r;
     }
 
     static __device__ __forceinline__ void issue_row(const RoundArgs &A, int k, unsigned char *buf, uint64_t *bars,
@@ -634,15 +660,15 @@ struct Round {
                 const int j = group_of(k, nt);
                 if (t == (k >> 3) - nt * j) xm ^= (M)1 << (8 * j + (k & 7));  // x_k <- 1 - x_k
             }
-            int vmin, cmin;
+            int vmin, cmin, cj;
             const uint4 *row4 = reinterpret_cast<const uint4 *>(row);
             M mism = 0;
             if (straight) {
                 mism = xm ^ stm[t];
-                process_row<kStraight>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
+                process_row<kStraight>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, cmin, cj);
             } else {
-                if (exact) process_row<kMin>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
-                else process_row<kUpdate>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin);
+                if (exact) process_row<kMin>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin, cj);
+                else process_row<kUpdate>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin, cj);
                 if (!sa) {
                     a += l;  // offset <- (a + l) mod n
                     if (a >= n) a -= n;
@@ -703,7 +729,7 @@ struct Round {
             if (improve || sidx) {
                 int it = INT_MAX, is = INT_MAX;
                 if (improve && r1.v < 0 && vmin == r1.v) it = lowest_equal(g, xm, ~(M)0, r1.v, t, nt);
-                if (sidx && cmin == r1.c) is = lowest_equal(g, xm, mism, r1.c, t, nt);
+                if (sidx && cmin == r1.c) is = lowest_equal_group(g, xm, mism, r1.c, cj, t, nt);
                 const Red r2 = block_reduce(Red{it, is, is}, sm->red, rb, lane, warp, nw);
                 if (improve) {
                     M bm = xm;
