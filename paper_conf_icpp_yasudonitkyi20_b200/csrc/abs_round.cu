@@ -117,6 +117,7 @@ struct RoundSmem {
     unsigned long long sa_ctr;  // SA: proposals drawn (Philox counter); thread 0 writes
     int sa_tau;                 // SA: this search's temperature
     int sa_d[2], sa_x[2];       // SA: Delta_k / x_k of the proposal, by counter parity
+    int snext[2];               // straight phase: 2k + x of the next flip, from its owner thread
 #ifdef ABS_TIMING
     long long tacc[32][24];  // [warp][local 0-6 | straight 8-14 | selection sub-phases 16-20]
 #endif
@@ -675,7 +676,10 @@ struct Round {
                 }
             }
             ABS_T(long long tc3 = clock64();)
-            int ci2 = INT_MAX;
+            // straight phase: the byte-group beta = t + nt * cj of this thread's first
+            // minimum; the CTA minimum of (cmin, beta) names the owner of the lowest-index
+            // argmin over the mismatches (i = 8 beta + e, reading C5)
+            int ci2 = (straight && cmin != INT_MAX) ? t + nt * cj : INT_MAX;
             if (!straight) {
                 if (pre) {
                     int a2 = a + l;
@@ -726,25 +730,50 @@ struct Round {
                 if (improve) sm->EB = sm->E + min(r1.v, 0);
             }
             const bool sidx = straight && r1.c != INT_MAX;
-            if (improve || sidx) {
-                int it = INT_MAX, is = INT_MAX;
-                if (improve && r1.v < 0 && vmin == r1.v) it = lowest_equal(g, xm, ~(M)0, r1.v, t, nt);
-                if (sidx && cmin == r1.c) is = lowest_equal_group(g, xm, mism, r1.c, cj, t, nt);
-                const Red r2 = block_reduce(Red{it, is, is}, sm->red, rb, lane, warp, nw);
-                if (improve) {
-                    M bm = xm;
-                    if (r1.v < 0) {
-                        const int istar = r2.v >> 1;
-                        const int j = group_of(istar, nt);
-                        if (t == (istar >> 3) - nt * j) bm ^= (M)1 << (8 * j + (istar & 7));
+            int snext = 0;
+            if (sidx) {
+                // The owner of byte-group beta finds the index in its 8 slots, publishes it
+                // (its warp arrives on named barrier 1, the other warps wait there) and
+                // issues the TMA for the next row: no second CTA reduction on the chain.
+                const int beta = r1.i;
+                const int jb = group_of(8 * beta, nt);
+                const int owner = beta - nt * jb;
+                if (!kMulti) {
+                    if (t == owner) {
+                        snext = lowest_equal_group(g, xm, mism, r1.c, jb, t, nt);
+                        sm->snext[b] = snext;
+                        issue_row(A, snext >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
                     }
-                    sbm[t] = bm;
+                    __syncwarp();
+                    snext = sm->snext[b];
+                } else if (warp == (owner >> 5)) {
+                    if (t == owner) {
+                        snext = lowest_equal_group(g, xm, mism, r1.c, jb, t, nt);
+                        sm->snext[b] = snext;
+                    }
+                    snext = __shfl_sync(kFull, snext, owner & 31);
+                    named_arrive(1, nt);
+                    if (t == owner) issue_row(A, snext >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+                } else {
+                    named_sync(1, nt);
+                    snext = sm->snext[b];
                 }
-                if (sidx) {
-                    k = r2.c >> 1;
-                    xk = r2.c & 1;
-                    dk = r1.c;
+            }
+            if (improve) {
+                M bm = xm;
+                if (r1.v < 0) {  // B = X' with its best neighbour flipped (reading C2)
+                    const int it = (vmin == r1.v) ? lowest_equal(g, xm, ~(M)0, r1.v, t, nt) : INT_MAX;
+                    const Red r2 = block_reduce(Red{it, INT_MAX, INT_MAX}, sm->red, rb, lane, warp, nw);
+                    const int istar = r2.v >> 1;
+                    const int j = group_of(istar, nt);
+                    if (t == (istar >> 3) - nt * j) bm ^= (M)1 << (8 * j + (istar & 7));
                 }
+                sbm[t] = bm;
+            }
+            if (sidx) {
+                k = snext >> 1;
+                xk = snext & 1;
+                dk = r1.c;
             }
 
             // ---- next flip
@@ -811,7 +840,7 @@ struct Round {
                 dk = r.c;
                 exact = true;
             }
-            if (t == ctl) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+            if (t == ctl && !sidx) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
             ABS_T(if (lane == 0) {
                 const long long tc6 = clock64();
                 sm->tacc[warp][to + 0] += tc1 - tc0;  // window selection (control warp)

@@ -46,4 +46,16 @@ __device__ __forceinline__ void mbar_wait(uint64_t *bar, uint32_t parity)
         : "memory");
 }
 
+// Named barriers (id >= 1; 0 is __syncthreads): `count` threads, a multiple of 32,
+// warp-uniform participation.  A producer warp writes shared memory, then arrives;
+// consumer warps sync, then read.
+__device__ __forceinline__ void named_sync(int id, int count)
+{
+    asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+__device__ __forceinline__ void named_arrive(int id, int count)
+{
+    asm volatile("bar.arrive %0, %1;" ::"r"(id), "r"(count) : "memory");
+}
+
 }  // namespace absb
