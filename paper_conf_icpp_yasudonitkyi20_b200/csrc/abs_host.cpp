@@ -127,6 +127,29 @@ static void ga_target(const Pool &P, const GaParams &ga, int64_t r, int64_t sid,
     }
 }
 
+// Run f(i) for i in [0, count) on up to min(16, cores) host threads; serial below
+// `grain` items.  Used for the GA targets of a lockstep step, which only READ the pool
+// (each target is a function of the pool, the round and the search id alone).
+template <class F>
+static void parallel_for(int count, int grain, const F &f)
+{
+    const int hc = (int)std::max(1u, std::thread::hardware_concurrency());
+    const int nth = std::min(std::min(16, hc), std::max(1, count / std::max(1, grain)));
+    if (nth <= 1) {
+        for (int i = 0; i < count; ++i) f(i);
+        return;
+    }
+    std::vector<std::thread> th;
+    th.reserve(nth - 1);
+    auto chunk = [&](int w) {
+        const int lo = (int)((int64_t)count * w / nth), hi = (int)((int64_t)count * (w + 1) / nth);
+        for (int i = lo; i < hi; ++i) f(i);
+    };
+    for (int w = 1; w < nth; ++w) th.emplace_back(chunk, w);
+    chunk(0);
+    for (auto &x : th) x.join();
+}
+
 }  // namespace absb
 
 using namespace absb;
@@ -433,12 +456,13 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
 static int lockstep_step(abs_ctx *c)
 {
     const int S = c->S.S, words = c->pool.words, bpv = c->bytes_per_vec;
-    // host Step 4: "generates ... new target solutions by GA"
+    // host Step 4: "generates ... new target solutions by GA"; the targets are
+    // independent given the pool, so large batches are built on several host threads
     std::vector<uint32_t> T(words);
-    for (int s = 0; s < S; ++s) {
-        ga_target(c->pool, c->ga, c->round, (int64_t)c->cfg.search_offset + s, T.data());
-        std::memcpy(c->T_h + (size_t)s * bpv, T.data(), sizeof(uint32_t) * words);
-    }
+    parallel_for(S, 512, [&](int s) {  // T_h rows: bpv = n_pad / 8 bytes, 4-byte aligned
+        ga_target(c->pool, c->ga, c->round, (int64_t)c->cfg.search_offset + s,
+                  reinterpret_cast<uint32_t *>(c->T_h + (size_t)s * bpv));
+    });
     ABS_CU(cudaMemcpyAsync(c->S.T, c->T_h, (size_t)S * bpv, cudaMemcpyHostToDevice, c->st));
     c->h2d += (int64_t)S * bpv;
     RoundArgs a{};
