@@ -131,6 +131,11 @@ template <int kP, int kMaxT, int kNT, bool kSA>
 struct Round {
     static constexpr int G = kP / 8;  // byte-groups per thread
     static constexpr bool kMulti = kMaxT > 32;
+    // B's neighbour bit i* from the owner of the byte-group the reduction names
+    // (no second reduction); else every thread scans its slots and a second
+    // reduction picks the lowest index
+    // (multi-warp kernels: measured slower at n = 32k, code generation of the flip loop)
+    static constexpr bool kOwnerB = !kMulti;
     using M = typename MaskOf<kP>::T;
 
     // ---------------------------------------------------------------- small helpers
@@ -263,12 +268,19 @@ struct Round {
 
     // CTA-wide min reduction (three keys); all threads get the result.  Lowest
     // index wins ties (reading C5).  Alternating slots -> one barrier per call.
-    static __device__ __forceinline__ Red block_reduce(Red r, Red (*sred)[32], int &rb, int lane, int warp, int nw)
+    // kOwnerB: vb = lowest byte-group holding a bit whose Delta is the minimum v
+    // (rvb: this thread's first such group, INT_MAX if none).
+    static __device__ __forceinline__ Red block_reduce(Red r, Red (*sred)[32], int &rb, int lane, int warp, int nw,
+                                                       int rvb = INT_MAX, int *vb = nullptr)
     {
         Red w;
         w.v = __reduce_min_sync(kFull, r.v);
         w.c = __reduce_min_sync(kFull, r.c);
         w.i = __reduce_min_sync(kFull, r.c == w.c ? r.i : INT_MAX);
+        if constexpr (kOwnerB) {
+            static_assert(!kMulti, "byte-group of the minimum: one-warp searches only");
+            if (vb) *vb = __reduce_min_sync(kFull, r.v == w.v ? rvb : INT_MAX);
+        }
         if (!kMulti) {
             __syncwarp();  // orders lane 0's shared-memory bookkeeping before other lanes read it
             return w;
@@ -307,18 +319,20 @@ struct Round {
 
     // Row update for one flip: g += c * W_k* over the P slots (Eq.(16), field
     // form), then, unless kMode == kUpdate, the n neighbour deltas (Eq.(5)):
-    // min over all bits (vmin) and, kMode == kStraight, over the mismatches (cmin).
+    // min over all bits (vmin) and, kMode == kStraight, over the mismatches (cmin);
+    // vj / cj: the first of this thread's byte-groups holding vmin / cmin.
     template <int kMode>
     static __device__ __forceinline__ void process_row(int (&g)[kP], M xm, M mism, const uint4 *row4, uint64_t *bars,
-                                                       uint32_t par, int c, int t, int nt, int &vmin, int &cmin,
-                                                       int &cj)
+                                                       uint32_t par, int c, int t, int nt, int &vmin, int &vj,
+                                                       int &cmin, int &cj)
     {
         vmin = INT_MAX;
+        vj = 0;
         cmin = INT_MAX;
         cj = 0;  // kStraight: first byte-group holding cmin (lowest index, reading C5)
 #pragma unroll
         for (int j = 0; j < G; ++j) {
-            int gmin = INT_MAX;
+            int gmin = INT_MAX, gv = INT_MAX;
             if (kRowChunks == 2 ? (j % (G / 2) == 0) : (j == 0)) mbar_wait(&bars[kRowChunks == 2 ? j / (G / 2) : 0], par);
             const uint4 w4 = row4[t + nt * j];
             const uint32_t wv[4] = {w4.x, w4.y, w4.z, w4.w};
@@ -330,13 +344,18 @@ struct Round {
                 if (kMode != kUpdate) {
                     const int d0 = readout(g[s0], xm, s0);
                     const int d1 = readout(g[s0 + 1], xm, s0 + 1);
-                    vmin = min(vmin, min(d0, d1));
+                    if (kOwnerB) gv = min(gv, min(d0, d1));
+                    else vmin = min(vmin, min(d0, d1));
                     if (kMode == kStraight) {
                         const int m0 = bit(mism, s0) ? d0 : INT_MAX;
                         const int m1 = bit(mism, s0 + 1) ? d1 : INT_MAX;
                         gmin = min(gmin, min(m0, m1));
                     }
                 }
+            }
+            if (kOwnerB && kMode != kUpdate && gv < vmin) {
+                vmin = gv;
+                vj = j;
             }
             if (kMode == kStraight && gmin < cmin) {
                 cmin = gmin;
@@ -661,15 +680,15 @@ struct Round {
                 const int j = group_of(k, nt);
                 if (t == (k >> 3) - nt * j) xm ^= (M)1 << (8 * j + (k & 7));  // x_k <- 1 - x_k
             }
-            int vmin, cmin, cj;
+            int vmin, vj, cmin, cj;
             const uint4 *row4 = reinterpret_cast<const uint4 *>(row);
             M mism = 0;
             if (straight) {
                 mism = xm ^ stm[t];
-                process_row<kStraight>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, cmin, cj);
+                process_row<kStraight>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, vj, cmin, cj);
             } else {
-                if (exact) process_row<kMin>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin, cj);
-                else process_row<kUpdate>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin, cj);
+                if (exact) process_row<kMin>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, vj, cmin, cj);
+                else process_row<kUpdate>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, vj, cmin, cj);
                 if (!sa) {
                     a += l;  // offset <- (a + l) mod n
                     if (a >= n) a -= n;
@@ -715,8 +734,10 @@ struct Round {
 
             ABS_T(long long tc4 = clock64();)
             Red r1;
+            int r1vb = INT_MAX;  // kOwnerB: byte-group of the lowest bit attaining r1.v
             if (exact || (!kMulti && !pre)) {  // one warp: the next window argmin is reduced here too
-                r1 = block_reduce(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw);
+                r1 = block_reduce(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw,
+                                  vmin != INT_MAX ? t + nt * vj : INT_MAX, &r1vb);
             } else {
                 sync();  // row buffer b free; sel[b], thr[b] and the window published
                 r1 = Red{INT_MAX, INT_MAX, INT_MAX};
@@ -759,14 +780,25 @@ struct Round {
                     snext = sm->snext[b];
                 }
             }
+            ABS_T(if (lane == 0 && straight) { sm->tacc[warp][7] += improve; sm->tacc[warp][15] += improve && r1.v < 0; })
             if (improve) {
                 M bm = xm;
                 if (r1.v < 0) {  // B = X' with its best neighbour flipped (reading C2)
-                    const int it = (vmin == r1.v) ? lowest_equal(g, xm, ~(M)0, r1.v, t, nt) : INT_MAX;
-                    const Red r2 = block_reduce(Red{it, INT_MAX, INT_MAX}, sm->red, rb, lane, warp, nw);
-                    const int istar = r2.v >> 1;
-                    const int j = group_of(istar, nt);
-                    if (t == (istar >> 3) - nt * j) bm ^= (M)1 << (8 * j + (istar & 7));
+                    if constexpr (kOwnerB) {
+                        // the reduction named the lowest byte-group holding the minimum; its owner
+                        // finds the lowest bit i* in its 8 slots and flips it in its part of B
+                        const int jv = group_of(8 * r1vb, nt);
+                        if (t == r1vb - nt * jv) {
+                            const int istar = lowest_equal_group(g, xm, ~(M)0, r1.v, jv, t, nt) >> 1;
+                            bm ^= (M)1 << (8 * jv + (istar & 7));
+                        }
+                    } else {
+                        const int it = (vmin == r1.v) ? lowest_equal(g, xm, ~(M)0, r1.v, t, nt) : INT_MAX;
+                        const Red r2 = block_reduce(Red{it, INT_MAX, INT_MAX}, sm->red, rb, lane, warp, nw);
+                        const int istar = r2.v >> 1;
+                        const int j = group_of(istar, nt);
+                        if (t == (istar >> 3) - nt * j) bm ^= (M)1 << (8 * j + (istar & 7));
+                    }
                 }
                 sbm[t] = bm;
             }

@@ -35,6 +35,10 @@ for kind, o in (("local", 0), ("straight", 8)):
         if nw > 1 else None,
         "control_warp": {nm: round(float(T[:, -1, o + i].sum() / fl[:, -1].sum()), 1) for i, nm in enumerate(names)},
     }
+if T[:, :, 14].sum() > 0:  # straight flips that improved E_B (control warp's count)
+    fl = T[:, -1, 14].sum()
+    out["straight_improve"] = {"fraction": float(T[:, -1, 7].sum() / fl),
+                               "fraction_neighbour": float(T[:, -1, 15].sum() / fl)}
 sub = T[:, -1, 16:21]
 if sub[:, 4].sum() > 0:
     out["selection_subphases"] = {nm: round(float(sub[:, i].sum() / sub[:, 4].sum()), 1) for i, nm in
