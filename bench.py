@@ -62,13 +62,22 @@ def make_W(workload: str):
     raise ValueError(workload)
 
 
+# Waves of co-resident searches per step.  A lockstep step ends with its
+# slowest search (straight-search lengths differ per target); with several
+# waves an SM whose search finishes early starts another.  Measured on one
+# B200: random32k 1/2/4/8 waves 2.49/2.52/2.59/2.61e12,
+# tsp100 1/4 waves 1.93/2.01e12; maxcut2k already runs 16 searches per SM.
+WAVES = {"random32k": 4, "tsp100": 4}
+
+
 def default_searches(workload: str, n: int, device: int) -> int:
-    """Config 2 fixes 10k searches at n=1024; elsewhere the searches whose
-    CTAs are co-resident on the GPU (148 at n=32k: one 512-thread CTA per SM)."""
+    """Config 2 fixes 10k searches at n=1024; elsewhere WAVES x the searches
+    whose CTAs are co-resident on the GPU (148 at n=32k: one 512-thread CTA
+    per SM)."""
     if workload == "random1k":
         return 10000
     import paper_conf_icpp_yasudonitkyi20_b200 as pkg
-    return pkg.device_searches(n, device)
+    return WAVES.get(workload, 1) * pkg.device_searches(n, device)
 
 
 # ------------------------------------------------------------------ clocks

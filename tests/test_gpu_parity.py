@@ -6,6 +6,8 @@ final pool."""
 from __future__ import annotations
 
 import itertools
+import os
+import sys
 import time
 
 import numpy as np
@@ -249,9 +251,9 @@ def test_seed_pool_uses_device_energies():
 
 # ---------------------------------------------------------------- full size (bench launch configuration)
 def test_full_size_n32768_sampled():
-    """n = 32768 (config 5) in the launch configuration bench.py times
-    (one 1024-thread CTA per search), on 2 sampled searches with a reduced
-    L: trajectory hash, Delta, E, B, E_B identical to the oracle."""
+    """n = 32768 (config 5), the kernel variant bench.py times (one 512-thread
+    CTA per search, 64 bits per thread), on 2 searches with a reduced L:
+    trajectory hash, Delta, E, B, E_B identical to the oracle."""
     n, S, L = 32768, 2, 64
     W = random_qubo(n, 1)
     t0 = time.time()
@@ -266,6 +268,46 @@ def test_full_size_n32768_sampled():
         assert st["E"] == o["E"][i]
         assert (st["D"].astype(np.int64) == o["D"][i]).all()
     assert time.time() - t0 < 600
+
+
+def test_bench_configuration_random32k_sampled():
+    """The exact step bench.py times by default: its W (random32k), seed, pool,
+    searches (WAVES x co-resident CTAs) and L = n, one lockstep step.  Three
+    sampled searches are re-run by the oracle from the oracle's own round-0
+    targets (host GA): E_B, B, final E, Delta, flip count and
+    trajectory hash identical."""
+    import threading
+
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+
+    W = bench.make_W("random32k")
+    n = W.shape[0]
+    S = bench.default_searches("random32k", n, 0)
+    s = make(W, searches=S, local_flips=n, pool_size=64, seed=1)
+    s.search(1)
+    B, EB = s.round_results()
+    cfg = ocfg(n, S, n, 64, 1)
+    pool = oracle.Pool(n, 64, 1)
+    lad = oracle.default_ladder(n)
+    sids = [0, S // 2 + 1, S - 1]
+    reps = {}
+
+    def replay(sid):
+        reps[sid] = oracle.replay_search(W, lad[sid % len(lad)], n, pool.target(cfg, 0, sid))
+
+    th = [threading.Thread(target=replay, args=(sid,)) for sid in sids]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join()
+    for sid in sids:
+        rep, st = reps[sid], s.search_state(sid)
+        assert EB[sid] == rep["EB"][0] and (B[sid] == rep["B"][0]).all()
+        assert st["hash"] == int(rep["hash"][0]) and st["flips"] == int(rep["flips"][0])
+        assert st["E"] == int(rep["E"][0]) and (st["X"] == rep["X"]).all()
+        assert (st["D"].astype(np.int64) == rep["D"]).all()
+    assert s.stats()["flips"] >= S * n
 
 
 # ---------------------------------------------------------------- asynchronous mode (paper Fig. 5)

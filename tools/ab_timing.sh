@@ -12,5 +12,5 @@ a=json.load(open('gpurun_out/timing_new.txt')); b=json.load(open('gpurun_out/tim
 for ph in ('local','straight'):
     for w in ('row_warps','control_warp'):
         print(ph, w, 'new', a[ph][w]); print(ph, w, 'old', b[ph][w])
-print(a.get('straight_improve'))
+print(a.get('straight_improve'), a.get('certain_selection_fraction'), a.get('selection_subphases'), b.get('selection_subphases'))
 PY

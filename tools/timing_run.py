@@ -39,6 +39,8 @@ if T[:, :, 14].sum() > 0:  # straight flips that improved E_B (control warp's co
     fl = T[:, -1, 14].sum()
     out["straight_improve"] = {"fraction": float(T[:, -1, 7].sum() / fl),
                                "fraction_neighbour": float(T[:, -1, 15].sum() / fl)}
+if T[:, -1, 20].sum() > 0 and T[:, -1, 21].sum() > 0:  # certain window selections (prefetch path)
+    out["certain_selection_fraction"] = float(T[:, -1, 21].sum() / T[:, -1, 20].sum())
 sub = T[:, -1, 16:21]
 if sub[:, 4].sum() > 0:
     out["selection_subphases"] = {nm: round(float(sub[:, i].sum() / sub[:, 4].sum()), 1) for i, nm in
