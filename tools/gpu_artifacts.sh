@@ -17,7 +17,7 @@ timeout 600 python bench.py --impl reference > $OUT/bench_ref.json 2> $OUT/bench
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
     python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > $OUT/bench_under_ncu.log 2>&1; echo "ncu-launches rc=$?"
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:round_kernel -s 2 -c 1 \
-    -o $OUT/prof_round python tools/prof_round.py --n 32768 --steps 3 > $OUT/prof_round.log 2>&1; echo "ncu-full rc=$?"
+    -o $OUT/prof_round python tools/prof_round.py --n 32768 --searches 592 --steps 3 > $OUT/prof_round.log 2>&1; echo "ncu-full rc=$?"
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:round_kernel -s 2 -c 1 \
     -o $OUT/prof_round1k python tools/prof_round.py --n 1024 --searches 10000 --steps 3 > $OUT/prof_round1k.log 2>&1; echo "ncu-full-1k rc=$?"
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:init_mma -s 2 -c 1 \
