@@ -66,6 +66,7 @@ struct MaskOf<64> {
 };
 
 constexpr uint32_t kTagSA = 0x5341504Cu;  // 'SAPL'
+constexpr int kSaBatch = 8;               // SA proposals evaluated per barrier (<= 32)
 
 // Philox4x32-10 (Salmon et al., SC'11), the library's device copy (the oracle
 // has its own; both are pinned by the Random123 known-answer vectors).
@@ -116,7 +117,7 @@ struct RoundSmem {
     long long nflip, nstraight;
     unsigned long long sa_ctr;  // SA: proposals drawn (Philox counter); thread 0 writes
     int sa_tau;                 // SA: this search's temperature
-    int sa_d[2], sa_x[2];       // SA: Delta_k / x_k of the proposal, by counter parity
+    int sa_d[2][8], sa_x[2][8]; // SA: Delta_k / x_k of a batch of proposals, by batch parity
     int snext[2];               // straight phase: 2k + x of the next flip, from its owner thread
 #ifdef ABS_TIMING
     long long tacc[32][24];  // [warp][local 0-6 | straight 8-14 | selection sub-phases 16-20]
@@ -326,6 +327,7 @@ struct Round {
                                                        uint32_t par, int c, int t, int nt, int &vmin, int &vj,
                                                        int &cmin, int &cj)
     {
+        const int cb = c & 0xff;  // c = +-2 as a signed byte
         vmin = INT_MAX;
         vj = 0;
         cmin = INT_MAX;
@@ -339,8 +341,11 @@ struct Round {
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
                 const int s0 = 8 * j + 2 * q;
-                g[s0] += c * sext16(wv[q]);
-                g[s0 + 1] += c * (((int)wv[q]) >> 16);
+                // g += c * W_ik for the two int16 of one word: one 2-way int16 x int8
+                // dot product each (IDP.2A on the FMA pipe; no sign-extension on the ALU
+                // pipe), with c in byte 0 (low half) or byte 1 (high half) of cb
+                g[s0] = __dp2a_lo((int)wv[q], cb, g[s0]);
+                g[s0 + 1] = __dp2a_lo((int)wv[q], cb << 8, g[s0 + 1]);
                 if (kMode != kUpdate) {
                     const int d0 = readout(g[s0], xm, s0);
                     const int d1 = readout(g[s0 + 1], xm, s0 + 1);
@@ -439,45 +444,77 @@ struct Round {
     }
 
     // SA policy (Alg. 1 + Eq.(7), reading E2): draw proposals until one is
-    // accepted or the round's proposal budget `left` is spent.  The owner of
-    // bit k broadcasts Delta_k and x_k through shared memory (slot = counter
-    // parity, one barrier per proposal).  Returns false when nothing was accepted.
+    // accepted or the round's proposal budget `left` is spent.  Proposals are
+    // evaluated in batches against the current state: lane q of every warp
+    // draws proposal c + q (Philox), the owners of the proposed bits broadcast
+    // Delta_k and x_k through shared memory (one barrier per batch), and lane q
+    // decides proposal q.  The first accepted one is taken; the proposals after
+    // it are discarded and drawn again after the flip, so the sequence of
+    // decisions is exactly the one-at-a-time sequence (rejections do not change
+    // the state).  The batch size bsz adapts to the acceptance rate (uniform
+    // across the CTA): doubled after a batch without acceptance, halved when
+    // the first proposal of a batch is accepted.  Returns false when nothing
+    // was accepted.
     static __device__ __forceinline__ bool sa_next(const RoundArgs &A, RoundSmem *sm, const int (&g)[kP], M xm,
-                                                   int sid, int n, int t, int nt, int &left, int &k, int &dk, int &xk)
+                                                   int sid, int n, int t, int nt, int &left, int &k, int &dk, int &xk,
+                                                   int &bsz)
     {
         unsigned long long c = sm->sa_ctr;  // written by thread 0 before the last barrier
         const int tau = sm->sa_tau;
         const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
+        const int lane = t & 31;
         bool acc = false;
+        int sb = 0;  // batch slot parity (a barrier separates this call from the previous one)
         while (left > 0) {
-            --left;
-            uint32_t o[4];
-            philox4x32_10((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
-            const int par = (int)(c & 1u);
-            ++c;
-            const int kk = (int)(o[0] % (uint32_t)n);  // "randomly select a bit" (Alg. 1)
-            const int j = group_of(kk, nt);
-            if (t == (kk >> 3) - nt * j) {
-                const int e = kk & 7;
-                int v = 0;
+            const int nb = min(left, bsz);
+            int kq = 0;
+            uint32_t o1 = 0;
+            if (lane < nb) {
+                uint32_t o[4];
+                const unsigned long long cq = c + (unsigned long long)lane;
+                philox4x32_10((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
+                kq = (int)(o[0] % (uint32_t)n);  // "randomly select a bit" (Alg. 1)
+                o1 = o[1];
+            }
+            for (int q = 0; q < nb; ++q) {
+                const int kk = __shfl_sync(kFull, kq, q);
+                const int j = group_of(kk, nt);
+                if (t == (kk >> 3) - nt * j) {
+                    const int e = kk & 7;
+                    int v = 0;
 #pragma unroll
-                for (int jj = 0; jj < G; ++jj)
+                    for (int jj = 0; jj < G; ++jj)
 #pragma unroll
-                    for (int ee = 0; ee < 8; ++ee)
-                        if (jj == j && ee == e) v = g[8 * jj + ee];
-                sm->sa_d[par] = readout(v, xm, 8 * j + e);
-                sm->sa_x[par] = (int)bit(xm, 8 * j + e);
+                        for (int ee = 0; ee < 8; ++ee)
+                            if (jj == j && ee == e) v = g[8 * jj + ee];
+                    sm->sa_d[sb][q] = readout(v, xm, 8 * j + e);
+                    sm->sa_x[sb][q] = (int)bit(xm, 8 * j + e);
+                }
             }
             sync();
-            const int d = sm->sa_d[par];
-            const int x = sm->sa_x[par];
-            if (d <= 0 || (uint64_t)o[1] < sa_threshold(d, tau)) {  // Eq.(7)
-                k = kk;
-                dk = d;
-                xk = x;
+            int d = 0, x = 0;
+            bool ok = false;
+            if (lane < nb) {
+                d = sm->sa_d[sb][lane];
+                x = sm->sa_x[sb][lane];
+                ok = d <= 0 || (uint64_t)o1 < sa_threshold(d, tau);  // Eq.(7)
+            }
+            const unsigned m = __ballot_sync(kFull, ok);
+            if (m) {
+                const int q = __ffs(m) - 1;  // the first accepted proposal
+                if (q == 0) bsz = max(1, bsz >> 1);
+                k = __shfl_sync(kFull, kq, q);
+                dk = __shfl_sync(kFull, d, q);
+                xk = __shfl_sync(kFull, x, q);
+                left -= q + 1;
+                c += (unsigned long long)(q + 1);
                 acc = true;
                 break;
             }
+            left -= nb;
+            c += (unsigned long long)nb;
+            sb ^= 1;
+            bsz = min(2 * bsz, kSaBatch);
         }
         if (t == 0) sm->sa_ctr = c;
         return acc;
@@ -558,6 +595,7 @@ struct Round {
         constexpr bool sa = kSA;  // ABS_POLICY_SA: a separate kernel instantiation
         const bool pre = kMulti && l <= kWinMax && !sa;
         int left = (int)A.L;
+        int sa_bsz = 1;  // SA: proposals per batch (sa_next)
         int rb = 0;
         sync();
 
@@ -566,7 +604,7 @@ struct Round {
         int k = 0, dk = 0, xk = 0;
         bool have = true;  // a first flip exists (SA may accept nothing)
         if (sa && !straight) {
-            have = sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk);
+            have = sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz);
         } else {
             int cv, ci2;
             if constexpr (kMulti) {  // one inlined scan (code size of the flip loop)
@@ -810,7 +848,7 @@ struct Round {
 
             // ---- next flip
             if (!straight && sa) {
-                if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk)) break;
+                if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz)) break;
                 if constexpr (!kMulti) {
                     __syncwarp();
                     const long long E1 = sm->E;
@@ -853,7 +891,7 @@ struct Round {
                 straight = false;
                 if (left <= 0) break;
                 if (sa) {
-                    if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk)) break;
+                    if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz)) break;
                     exact = true;
                     if (t == ctl) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
                     continue;
