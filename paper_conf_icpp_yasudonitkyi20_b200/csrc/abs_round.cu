@@ -679,18 +679,17 @@ struct Round {
                             ww[q] = rw[i];
                         }
                     }
+                    // k_f is not in this window (windows are disjoint: l <= kWinMax <= n/8 here),
+                    // so every entry moves by Eq.(16); the four keys are reduced as a tree
+                    long long kq[4];
 #pragma unroll
                     for (int q = 0; q < 4; ++q) {
-                        if (lane + 32 * (4 * h + q) < l) {
-                            const int i = ii[q];
-                            const bool isk = i == k;
-                            const int w2 = (xx[q] == xk) ? 2 * ww[q] : -2 * ww[q];  // Eq.(16)
-                            const int d = isk ? -dd[q] : dd[q] + w2;                  // Eq.(6) at i = k
-                            const int xn = xx[q] ^ (int)isk;
-                            best = min(best, (long long)(((unsigned long long)(unsigned)d << 32) |
-                                                         (unsigned)(2 * i + xn)));
-                        }
+                        const int d = dd[q] + ww[q] * (2 - 4 * (xx[q] ^ xk));  // Eq.(16)
+                        kq[q] = (lane + 32 * (4 * h + q) < l)
+                                    ? (long long)(((unsigned long long)(unsigned)d << 32) | (unsigned)(2 * ii[q] + xx[q]))
+                                    : LLONG_MAX;
                     }
+                    best = min(best, min(min(kq[0], kq[1]), min(kq[2], kq[3])));
                 }
                 const int bv = (int)(best >> 32);
                 ABS_T(const long long ts2 = clock64();)
