@@ -13,6 +13,9 @@ timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err; echo "bench rc=
 for w in random1k maxcut2k tsp100; do
   timeout 600 python bench.py --workload $w --no-cpu-baseline > $OUT/bench_$w.json 2>> $OUT/bench.err; echo "bench $w rc=$?"
 done
+for w in random32k random1k maxcut2k; do
+  timeout 600 python bench.py --workload $w --policy sa --steps 3 --no-e2e --no-cpu-baseline > $OUT/sa_$w.json 2>> $OUT/bench.err; echo "sa $w rc=$?"
+done
 timeout 600 python bench.py --impl reference > $OUT/bench_ref.json 2> $OUT/bench_ref.err; echo "ref rc=$?"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
     python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > $OUT/bench_under_ncu.log 2>&1; echo "ncu-launches rc=$?"
