@@ -635,7 +635,7 @@ struct Round {
             unsigned char *row = rowbuf + rowb * b;
             ABS_T(long long tc0 = clock64(); const int to = straight ? 8 : 0;)
 
-            // ---- window-first selection of the next flip (warp 0), prefetch its row
+            // ---- window-first selection of the next flip (the last warp, the controller), prefetch its row
             if (pre && !straight && left > 1 && warp == nw - 1) {
                 int a1 = a + l;
                 if (a1 >= n) a1 -= n;
