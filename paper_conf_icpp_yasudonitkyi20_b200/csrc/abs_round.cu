@@ -392,7 +392,9 @@ struct Round {
                                                      int nt)
     {
         const uint32_t half = 8u * G * (uint32_t)nt;  // bytes of G/2 byte-groups = n_pad bytes
-        const char *src = reinterpret_cast<const char *>(A.Wz) + (size_t)k * (size_t)A.n_pad * 2;
+        // row stride 2 n_pad bytes; a compile-time constant when NT is (n = 32k: a shift)
+        const size_t stride = kNT ? (size_t)2 * kP * kNT : (size_t)A.n_pad * 2;
+        const char *src = reinterpret_cast<const char *>(A.Wz) + (size_t)k * stride;
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
             if (kRowChunks == 1) {
