@@ -698,10 +698,10 @@ struct Round {
                 const int mv = __reduce_min_sync(kFull, bv);
                 const int mi = __reduce_min_sync(kFull, bv == mv ? (int)(unsigned)best : INT_MAX);
                 ABS_T(const long long ts3 = clock64();)
-                if (lane == 0) {
-                    issue_row(A, mi >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
-                    sm->sel[b] = make_int4(mi >> 1, mv, mi & 1, 1);
-                }
+                // the warp is converged here: one elected lane issues (no per-lane loop
+                // around the bulk copy's uniform operands)
+                if (elect_one()) issue_row(A, mi >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+                if (lane == 0) sm->sel[b] = make_int4(mi >> 1, mv, mi & 1, 1);
                 ABS_T(if (lane == 0) {
                     const long long ts4 = clock64();
                     sm->tacc[warp][16] += ts1 - tc0;  // wait for row k_f's window half
