@@ -270,20 +270,21 @@ def test_full_size_n32768_sampled():
     assert time.time() - t0 < 600
 
 
-def test_bench_configuration_random32k_sampled():
-    """The exact step bench.py times by default: its W (random32k), seed, pool,
-    searches (WAVES x co-resident CTAs) and L = n, one lockstep step.  Three
-    sampled searches are re-run by the oracle from the oracle's own round-0
-    targets (host GA): E_B, B, final E, Delta, flip count and
-    trajectory hash identical."""
+@pytest.mark.parametrize("workload", ["random32k", "tsp100", "maxcut2k", "random1k"])
+def test_bench_configuration_sampled(workload):
+    """The exact step bench.py times by default for each workload: its W, seed,
+    pool, searches (WAVES x co-resident CTAs, or config 2's 10,000) and L = n,
+    one lockstep step.  Three sampled searches are re-run by the oracle from
+    the oracle's own round-0 targets (host GA): E_B, B, final E,
+    Delta, flip count and trajectory hash identical."""
     import threading
 
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import bench
 
-    W = bench.make_W("random32k")
+    W = bench.make_W(workload)
     n = W.shape[0]
-    S = bench.default_searches("random32k", n, 0)
+    S = bench.default_searches(workload, n, 0)
     s = make(W, searches=S, local_flips=n, pool_size=64, seed=1)
     s.search(1)
     B, EB = s.round_results()
