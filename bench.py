@@ -216,10 +216,19 @@ def run_abs(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
+    # test hooks for exercising the multi-rank flow on a single GPU (both ranks on
+    # one device, gloo for the exchange); the driver's runs use the defaults
+    local = int(os.environ.get("ABS_BENCH_DEVICE", local))
+    backend = os.environ.get("ABS_BENCH_BACKEND", "nccl")
     assert torch.cuda.is_available(), "bench.py needs B200 GPUs"
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+
+    rdev = "cuda" if backend == "nccl" else "cpu"  # device of the timing reductions
 
     def barrier():
         if world > 1:
@@ -277,8 +286,8 @@ def run_abs(args):
     kern_s = st1["search_seconds"] - st0["search_seconds"]
     launches = st1["round_kernel_launches"] - st0["round_kernel_launches"]
     all_launches = st1["kernel_launches"] - st0["kernel_launches"]
-    t_ms = torch.tensor([ms], dtype=torch.float64, device="cuda")
-    t_fl = torch.tensor([flips], dtype=torch.float64, device="cuda")
+    t_ms = torch.tensor([ms], dtype=torch.float64, device=rdev)
+    t_fl = torch.tensor([flips], dtype=torch.float64, device=rdev)
     if world > 1:
         dist.all_reduce(t_ms, op=dist.ReduceOp.MAX)
         dist.all_reduce(t_fl, op=dist.ReduceOp.SUM)
@@ -345,8 +354,8 @@ def run_abs(args):
         st2 = s2.stats()
         s2.close()
         ems = e0.elapsed_time(e1)
-        t2 = torch.tensor([ems], dtype=torch.float64, device="cuda")
-        f2 = torch.tensor([st2["flips"]], dtype=torch.float64, device="cuda")
+        t2 = torch.tensor([ems], dtype=torch.float64, device=rdev)
+        f2 = torch.tensor([st2["flips"]], dtype=torch.float64, device=rdev)
         if world > 1:
             dist.all_reduce(t2, op=dist.ReduceOp.MAX)
             dist.all_reduce(f2, op=dist.ReduceOp.SUM)
