@@ -118,6 +118,9 @@ struct RoundSmem {
     unsigned long long sa_ctr;  // SA: proposals drawn (Philox counter); thread 0 writes
     int sa_tau;                 // SA: this search's temperature
     int sa_d[2][8], sa_x[2][8]; // SA: Delta_k / x_k of a batch of proposals, by batch parity
+    int sa_k[2][8];             // SA: the batch's proposed bits ...
+    uint32_t sa_o[2][8];        // ... and their acceptance draws
+    int4 sa_e;                  // SA early decision of this flip: (k, Delta_k, x_k, proposals consumed)
     int snext[2];               // straight phase: 2k + x of the next flip, from its owner thread
 #ifdef ABS_TIMING
     long long tacc[32][24];  // [warp][local 0-6 | straight 8-14 | selection sub-phases 16-20]
@@ -457,11 +460,16 @@ struct Round {
     // across the CTA): doubled after a batch without acceptance, halved when
     // the first proposal of a batch is accepted.  Returns false when nothing
     // was accepted.
+    // The proposals of the accepted batch after the accepted one (lo_n of them,
+    // from index lo_q of slot lo_s) are left in shared memory for the next
+    // flip's early decision; cadd counts proposals that decision consumed.
     static __device__ __forceinline__ bool sa_next(const RoundArgs &A, RoundSmem *sm, const int (&g)[kP], M xm,
                                                    int sid, int n, int t, int nt, int &left, int &k, int &dk, int &xk,
-                                                   int &bsz)
+                                                   int &bsz, int &cadd, int &lo_n, int &lo_s, int &lo_q)
     {
-        unsigned long long c = sm->sa_ctr;  // written by thread 0 before the last barrier
+        unsigned long long c = sm->sa_ctr + (unsigned long long)cadd;  // thread 0 wrote sa_ctr before the last barrier
+        cadd = 0;
+        lo_n = 0;
         const int tau = sm->sa_tau;
         const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
         const int lane = t & 31;
@@ -477,6 +485,10 @@ struct Round {
                 philox4x32_10((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
                 kq = (int)(o[0] % (uint32_t)n);  // "randomly select a bit" (Alg. 1)
                 o1 = o[1];
+                if (t < 32) {
+                    sm->sa_k[sb][lane] = kq;
+                    sm->sa_o[sb][lane] = o1;
+                }
             }
             for (int q = 0; q < nb; ++q) {
                 const int kk = __shfl_sync(kFull, kq, q);
@@ -510,6 +522,9 @@ struct Round {
                 xk = __shfl_sync(kFull, x, q);
                 left -= q + 1;
                 c += (unsigned long long)(q + 1);
+                lo_n = nb - q - 1;
+                lo_s = sb;
+                lo_q = q + 1;
                 acc = true;
                 break;
             }
@@ -598,6 +613,7 @@ struct Round {
         const bool pre = kMulti && l <= kWinMax && !sa;
         int left = (int)A.L;
         int sa_bsz = 1;  // SA: proposals per batch (sa_next)
+        int sa_cadd = 0, sa_lon = 0, sa_los = 0, sa_loq = 0;  // SA: early decision bookkeeping (sa_next)
         int rb = 0;
         sync();
 
@@ -606,7 +622,7 @@ struct Round {
         int k = 0, dk = 0, xk = 0;
         bool have = true;  // a first flip exists (SA may accept nothing)
         if (sa && !straight) {
-            have = sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz);
+            have = sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq);
         } else {
             int cv, ci2;
             if constexpr (kMulti) {  // one inlined scan (code size of the flip loop)
@@ -710,6 +726,42 @@ struct Round {
                     sm->tacc[warp][19] += ts4 - ts3;  // TMA issue + sel
                     sm->tacc[warp][20] += 1;
                 })
+            }
+
+            // ---- SA early decision (the SA analogue of the window-first selection): the
+            // proposals left over from the batch that accepted k_f were drawn already;
+            // their Delta(X_{f+1}) needs one entry of row k_f each (Eq.(16)), so the
+            // controller decides them as soon as row k_f lands and, on an acceptance,
+            // issues the next row before the update.  Same decisions, in the same
+            // order, as one at a time (rejections do not change the state).
+            const int sa_cnt = (sa && !straight) ? min(sa_lon, left) : 0;  // uniform
+            if (sa_cnt > 0 && warp == nw - 1) {
+                mbar_wait(&sm->bar[b][0], par);
+                if (kRowChunks == 2) mbar_wait(&sm->bar[b][1], par);
+                int kk = 0, d = 0, xn = 0;
+                bool ok = false;
+                if (lane < sa_cnt) {
+                    const int q = sa_loq + lane;
+                    kk = sm->sa_k[sa_los][q];
+                    const uint32_t o1 = sm->sa_o[sa_los][q];
+                    const int d0 = sm->sa_d[sa_los][q];
+                    const int x0 = sm->sa_x[sa_los][q];
+                    if (kk == k) {  // Eq.(6): Delta_k(X') = -Delta_k(X)
+                        d = -d0;
+                        xn = x0 ^ 1;
+                    } else {
+                        d = d0 + reinterpret_cast<const short *>(row)[kk] * (2 - 4 * (x0 ^ xk));
+                        xn = x0;
+                    }
+                    ok = d <= 0 || (uint64_t)o1 < sa_threshold(d, sm->sa_tau);  // Eq.(7)
+                }
+                const unsigned m = __ballot_sync(kFull, ok);
+                const int j = m ? __ffs(m) - 1 : -1;
+                const int kn = __shfl_sync(kFull, kk, max(j, 0));
+                const int dn = __shfl_sync(kFull, d, max(j, 0));
+                const int xnn = __shfl_sync(kFull, xn, max(j, 0));
+                if (j >= 0 && elect_one()) issue_row(A, kn, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+                if (lane == 0) sm->sa_e = make_int4(j >= 0 ? kn : -1, dn, xnn, j >= 0 ? j + 1 : sa_cnt);
             }
 
             ABS_T(long long tc1 = clock64(); mbar_wait(&sm->bar[b][0], par); long long tc2 = clock64();)
@@ -849,7 +901,25 @@ struct Round {
 
             // ---- next flip
             if (!straight && sa) {
-                if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz)) break;
+                if (sa_cnt > 0) {  // this flip's early decision (written before the end-of-flip barrier)
+                    const int4 e = sm->sa_e;
+                    left -= e.w;
+                    sa_cadd += e.w;
+                    sa_lon = 0;
+                    if (e.x >= 0) {  // accepted: its row is in flight
+                        k = e.x;
+                        dk = e.y;
+                        xk = e.z;
+                        if constexpr (!kMulti) {
+                            __syncwarp();
+                            const long long E1 = sm->E;
+                            const long long LB2 = min(sm->LB - 2 * (long long)A.wmax, -(long long)dk);
+                            exact = E1 + dk + min(LB2, 0LL) < sm->EB;
+                        }
+                        continue;
+                    }
+                }
+                if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq)) break;
                 if constexpr (!kMulti) {
                     __syncwarp();
                     const long long E1 = sm->E;
@@ -892,7 +962,7 @@ struct Round {
                 straight = false;
                 if (left <= 0) break;
                 if (sa) {
-                    if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz)) break;
+                    if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq)) break;
                     exact = true;
                     if (t == ctl) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
                     continue;

@@ -67,6 +67,15 @@ def test_sa_lockstep_bitexact(n, S, L, R, seed):
     assert o["flips"].sum() > 0
 
 
+def test_sa_n32768_bench_variant():
+    """The kernel variant bench.py --policy sa times at n = 32768 (one
+    512-thread CTA per search), 2 searches, reduced L: bit-exact."""
+    n = 32768
+    W = random_qubo(n, 1)
+    s, o, gB, gEB = run_sa(W, 2, 400, 1, tmin=8000, tmax=262136, K=2, seed=1)
+    check(s, o, gB, gEB, 2, 8)
+
+
 def test_sa_maxcut_ties():
     n = 2000
     W = maxcut_qubo(n, 19990, seed=5)
