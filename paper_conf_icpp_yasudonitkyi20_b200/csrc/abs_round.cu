@@ -140,6 +140,9 @@ struct Round {
     // reduction picks the lowest index
     // (multi-warp kernels: measured slower at n = 32k, code generation of the flip loop)
     static constexpr bool kOwnerB = !kMulti;
+    // SA early decision (run()): off for one warp x 64 bits (n_pad = 2048), where it
+    // measured slower (MaxCut's high acceptance leaves few leftover proposals)
+    static constexpr bool kSaEarly = kSA && (kMulti || kP == 32);
     using M = typename MaskOf<kP>::T;
 
     // ---------------------------------------------------------------- small helpers
@@ -734,7 +737,7 @@ struct Round {
             // controller decides them as soon as row k_f lands and, on an acceptance,
             // issues the next row before the update.  Same decisions, in the same
             // order, as one at a time (rejections do not change the state).
-            const int sa_cnt = (sa && !straight) ? min(sa_lon, left) : 0;  // uniform
+            const int sa_cnt = (kSaEarly && !straight) ? min(sa_lon, left) : 0;  // uniform
             if (sa_cnt > 0 && warp == nw - 1) {
                 mbar_wait(&sm->bar[b][0], par);
                 if (kRowChunks == 2) mbar_wait(&sm->bar[b][1], par);
