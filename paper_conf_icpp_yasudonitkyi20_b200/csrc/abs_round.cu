@@ -1214,6 +1214,7 @@ int round_occupancy(int32_t nt, int32_t bpt, int *per_sm)
     }
     if (nt == 32) return occupancy_variant<64, 32, 32>(nt, smem, per_sm);  // n_pad = 2048
     if (nt == 512) return occupancy_variant<64, 512, 512>(nt, smem, per_sm);
+    if (nt == 160) return occupancy_variant<64, 512, 160>(nt, smem, per_sm);  // n_pad = 10240 (TSP, 100 cities)
     return occupancy_variant<64, 512, 0>(nt, smem, per_sm);
 }
 
@@ -1226,6 +1227,7 @@ int launch_round(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q, int *g
     }
     if (a.nt == 32) return launch_variant<64, 32, 32>(a, st, smem, q, grid_out);  // n_pad = 2048
     if (a.nt == 512) return launch_variant<64, 512, 512>(a, st, smem, q, grid_out);  // n_pad = 32768
+    if (a.nt == 160) return launch_variant<64, 512, 160>(a, st, smem, q, grid_out);  // n_pad = 10240 (TSP, 100 cities)
     return launch_variant<64, 512, 0>(a, st, smem, q, grid_out);
 }
 

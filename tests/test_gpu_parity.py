@@ -132,7 +132,8 @@ def test_config1_n16_bitexact_and_bruteforce():
     (1024, 6, 1024, 2, 3),     # config-2 size, one warp, full
     (1100, 5, 300, 2, 4),      # one warp, 64 bits per thread (n_pad 2048), ragged
     (3000, 4, 500, 2, 5),      # 3 warps
-    (4100, 3, 400, 2, 6),      # NT = 160
+    (4100, 3, 400, 2, 6),      # NT = 96 (runtime NT)
+    (10000, 3, 300, 2, 7),     # NT = 160 (compile-time NT: the TSP 100-city size)
 ])
 def test_lockstep_random_qubo_bitexact(n, S, L, R, seed):
     W = random_qubo(n, seed)

@@ -57,7 +57,8 @@ def check(s, o, gB, gEB, S, pool):
     (100, 8, 600, 3, 1),     # one warp, 32 bits per thread
     (1100, 5, 800, 2, 2),    # one warp, 64 bits per thread
     (3000, 4, 900, 2, 3),    # three warps
-    (4100, 3, 700, 2, 4),    # NT = 160
+    (4100, 3, 700, 2, 4),    # NT = 96 (runtime NT)
+    (10000, 2, 500, 1, 6),   # NT = 160 (compile-time NT: the TSP 100-city size)
 ])
 def test_sa_lockstep_bitexact(n, S, L, R, seed):
     W = random_qubo(n, seed)
