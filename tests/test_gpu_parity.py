@@ -388,3 +388,40 @@ def test_lockstep_short_local_phases(L):
     W = random_qubo(n, 60 + L)
     s, o, gB, gEB, gT = run_both(W, 4, L, 3, pool=8, seed=60 + L, ladder=[64, 256])
     assert_same(s, o, gB, gEB, 4, n, 8)
+
+
+def _degenerate_w(kind, n):
+    if kind == "zeros":        # every Delta is 0: every argmin is a full tie
+        return np.zeros((n, n), np.int16)
+    if kind == "minus_one":    # constant W = -1: ties in every window, E strictly falls
+        return np.full((n, n), -1, np.int16)
+    if kind == "diag_only":    # separable: the optimum sets exactly the negative diagonal bits
+        W = np.zeros((n, n), np.int16)
+        d = random_qubo(n, 71).diagonal()
+        W[np.arange(n), np.arange(n)] = d
+        return W
+    if kind == "extreme":      # +-32767/-32768 entries: the widest Delta range (reading C12)
+        rng = np.random.default_rng(72)
+        U = np.where(rng.random((n, n)) < 0.5, np.int16(-32768), np.int16(32767))
+        U = np.triu(U)
+        return (U + np.triu(U, 1).T).astype(np.int16)
+    return random_qubo(n, 73)
+
+
+@pytest.mark.parametrize("n,kind", [
+    (1, "random"), (2, "random"), (3, "minus_one"),   # smaller than one byte-group
+    (64, "zeros"), (200, "minus_one"), (500, "diag_only"),
+    (2048, "extreme"),      # one warp x 64 bits, n = n_pad exactly (no ragged tail)
+    (3072, "random"),       # 32 bits x 96 threads, n = n_pad exactly
+])
+def test_lockstep_degenerate_and_boundary(n, kind):
+    # degenerate instances (all ties, separable, extreme weights) and sizes at the
+    # edges of the kernel variants; trajectories, pool and every (B, E_B) bit-exact
+    W = _degenerate_w(kind, n)
+    S, L = 6, max(1, min(3 * n, 700))
+    s, o, gB, gEB, gT = run_both(W, S, L, 3, pool=8, seed=74)
+    assert_same(s, o, gB, gEB, S, n, 8)
+    if kind == "diag_only":
+        assert s.best()[1] == int(np.minimum(W.diagonal().astype(np.int64), 0).sum())
+    if kind == "zeros":
+        assert s.best()[1] == 0
