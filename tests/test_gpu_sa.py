@@ -105,3 +105,27 @@ def test_sa_async_emits_true_energies():
     assert len(E) > 0
     assert (s.energy(X) == E).all()
     s.close()
+
+
+@pytest.mark.parametrize("n,kind,tmin,tmax", [
+    (1, "random", 1, 1),             # a single bit; cold
+    (3, "random", 50000, 400000),    # smaller than one byte-group; hot
+    (64, "zeros", 1, 1),             # Delta = 0 everywhere: every proposal is accepted (d <= 0)
+    (500, "extreme", 1, 1),          # +-32767/-32768 entries, tau = 1: only downhill moves
+    (2048, "extreme", 2000, 2000000),  # one warp x 64 bits, n = n_pad exactly
+])
+def test_sa_degenerate_and_boundary(n, kind, tmin, tmax):
+    rng = np.random.default_rng(90 + n)
+    if kind == "zeros":
+        W = np.zeros((n, n), np.int16)
+    elif kind == "extreme":
+        U = np.triu(np.where(rng.random((n, n)) < 0.5, np.int16(-32768), np.int16(32767)))
+        W = (U + np.triu(U, 1).T).astype(np.int16)
+    else:
+        W = random_qubo(n, 91)
+    S, L = 4, max(1, min(20 * n, 900))
+    s, o, gB, gEB = run_sa(W, S, L, 3, tmin=tmin, tmax=tmax, K=2, seed=92)
+    check(s, o, gB, gEB, S, 8)
+    if kind == "zeros":
+        # every proposal accepted: exactly L flips per search and round after the straight phase
+        assert (o["flips"] >= 3 * L).all()
