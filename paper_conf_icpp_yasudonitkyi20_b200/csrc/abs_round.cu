@@ -66,7 +66,19 @@ struct MaskOf<64> {
 };
 
 constexpr uint32_t kTagSA = 0x5341504Cu;  // 'SAPL'
-constexpr int kSaBatch = 8;               // SA proposals evaluated per barrier (<= 32)
+// SA proposals evaluated per barrier (at most; the batch adapts, sa_next), <= 32 (one lane
+// per proposal).  Multi-warp searches (n > 2048) pay a CTA barrier per batch: 32 measured
+// +9.5% at n = 32k and +1.5% at n = 10,000 over 8.  One-warp searches keep 8: their CTAs
+// are small and many per SM, so the shared-memory bytes count (16 measured -1.5% at n = 1k).
+#ifndef ABS_SA_BATCH_ONE
+#define ABS_SA_BATCH_ONE 8
+#endif
+#ifndef ABS_SA_BATCH_MULTI
+#define ABS_SA_BATCH_MULTI 32
+#endif
+constexpr int kSaBatchOne = ABS_SA_BATCH_ONE, kSaBatchMulti = ABS_SA_BATCH_MULTI;
+static_assert(kSaBatchOne >= 1 && kSaBatchOne <= 32 && kSaBatchMulti >= 1 && kSaBatchMulti <= 32,
+              "one lane per proposal");
 
 // Philox4x32-10 (Salmon et al., SC'11), the library's device copy (the oracle
 // has its own; both are pinned by the Random123 known-answer vectors).
@@ -106,8 +118,9 @@ struct Red {
     int i;  // 2 * (lowest index attaining c) + x_index (INT_MAX if unknown / none)
 };
 
-// Shared-memory bookkeeping of a CTA (fixed size, at offset 0).
-struct RoundSmem {
+// Shared-memory bookkeeping of a CTA (at offset 0; kB = the SA batch cap).
+template <int kB>
+struct RoundSmemT {
     uint64_t bar[2][2];   // [row buffer][half row]
     Red red[2][32];
     int4 sel[2];          // window warp -> all: next (k, Delta_k, x_k, exact_next), by flip parity
@@ -117,9 +130,9 @@ struct RoundSmem {
     long long nflip, nstraight;
     unsigned long long sa_ctr;  // SA: proposals drawn (Philox counter); thread 0 writes
     int sa_tau;                 // SA: this search's temperature
-    int sa_d[2][8], sa_x[2][8]; // SA: Delta_k / x_k of a batch of proposals, by batch parity
-    int sa_k[2][8];             // SA: the batch's proposed bits ...
-    uint32_t sa_o[2][8];        // ... and their acceptance draws
+    int sa_d[2][kB], sa_x[2][kB];  // SA: Delta_k / x_k of a batch of proposals, by batch parity
+    int sa_k[2][kB];               // SA: the batch's proposed bits ...
+    uint32_t sa_o[2][kB];          // ... and their acceptance draws
     int4 sa_e;                  // SA early decision of this flip: (k, Delta_k, x_k, proposals consumed)
     int snext[2];               // straight phase: 2k + x of the next flip, from its owner thread
 #ifdef ABS_TIMING
@@ -135,6 +148,8 @@ template <int kP, int kMaxT, int kNT, bool kSA>
 struct Round {
     static constexpr int G = kP / 8;  // byte-groups per thread
     static constexpr bool kMulti = kMaxT > 32;
+    static constexpr int kSaBatch = kMulti ? kSaBatchMulti : kSaBatchOne;
+    using RoundSmem = RoundSmemT<kSaBatch>;
     // B's neighbour bit i* from the owner of the byte-group the reduction names
     // (no second reduction); else every thread scans its slots and a second
     // reduction picks the lowest index
@@ -1185,7 +1200,8 @@ size_t round_smem_bytes(int32_t nt, int32_t bpt)
 {
     const bool multi = nt > 32;
     const size_t msz = bpt == 64 ? 8 : 4;
-    size_t s = sizeof(RoundSmem) + (multi ? sizeof(WindowSmem) : 0) + 2 * msz * (size_t)nt;
+    size_t s = (multi ? sizeof(RoundSmemT<kSaBatchMulti>) + sizeof(WindowSmem) : sizeof(RoundSmemT<kSaBatchOne>)) +
+               2 * msz * (size_t)nt;
     s = (s + 127) & ~size_t(127);
     return s + 2 * (size_t)2 * bpt * nt;  // two row buffers of 2 * n_pad bytes
 }
