@@ -425,3 +425,74 @@ def test_lockstep_degenerate_and_boundary(n, kind):
         assert s.best()[1] == int(np.minimum(W.diagonal().astype(np.int64), 0).sum())
     if kind == "zeros":
         assert s.best()[1] == 0
+
+
+# ---------------------------------------------------------------- multi-warp kernels at the ladder extremes
+@pytest.mark.parametrize("n", [3000, 10000, 32768])
+def test_lockstep_multiwarp_ladder_extremes(n):
+    """Multi-warp kernels (n > 2048) with window lengths at both ends of
+    P:L305 (l = 1 ... l = n): l in {1, 2, 3} runs the window-first prefetch
+    path with windows shorter than a byte-group, l in {300, n/2+1, n} the
+    non-prefetch local branch (l > kWinMax = 256; for l > n/2 consecutive
+    windows overlap, l = n is steepest forced greedy).  Full state and every
+    (B, E_B) identical to oracle.run_lockstep."""
+    ladder = [1, 2, 3, 300, n // 2 + 1, n]
+    W = random_qubo(n, 80 + n % 97)
+    S, L, R = 6, 400, 2
+    s, o, gB, gEB, gT = run_both(W, S, L, R, pool=8, seed=81, ladder=ladder)
+    assert_same(s, o, gB, gEB, S, n, 8)
+
+
+def test_full_size_bench_three_rounds_replay():
+    """bench.py's default step (random n = 32768, 592 searches, L = n, seed 1)
+    for THREE lockstep steps.  (1) The host GA at full size: the targets of
+    rounds 1 and 2 equal oracle GA targets drawn from a pool rebuilt with
+    oracle.Pool from every result the device emitted.
+    (2) Three sampled searches are replayed by the oracle from the targets the
+    device used: every round's (B, E_B) and the final state identical."""
+    import threading
+
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import bench
+
+    W = bench.make_W("random32k")
+    n = W.shape[0]
+    S = bench.default_searches("random32k", n, 0)
+    s = make(W, searches=S, local_flips=n, pool_size=64, seed=1)
+    Ts, Bs, EBs = [], [], []
+    for _ in range(3):
+        s.search(1)
+        Ts.append(s.round_targets())
+        B, EB = s.round_results()
+        Bs.append(B)
+        EBs.append(EB)
+    cfg = ocfg(n, S, n, 64, 1)
+    pool = oracle.Pool(n, 64, 1)
+    for r in range(3):
+        for sid in [0, 1, S // 3, S - 1]:
+            assert (Ts[r][sid] == pool.target(cfg, r, sid)).all(), ("GA target", r, sid)
+        for sid in range(S):
+            pool.insert(Bs[r][sid], EBs[r][sid])
+    PX, PE = s.pool(64)
+    fin = pool.E != oracle.EINF
+    assert (PE == pool.E[fin]).all() and (PX == pool.X[fin]).all()
+
+    lad = oracle.default_ladder(n)
+    sids = [0, S // 2 + 1, S - 1]
+    reps = {}
+
+    def replay(sid):
+        reps[sid] = oracle.replay_search(W, lad[sid % len(lad)], n, np.stack([Ts[r][sid] for r in range(3)]))
+
+    th = [threading.Thread(target=replay, args=(sid,)) for sid in sids]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join()
+    for sid in sids:
+        rep, st = reps[sid], s.search_state(sid)
+        for r in range(3):
+            assert EBs[r][sid] == rep["EB"][r] and (Bs[r][sid] == rep["B"][r]).all(), ("round", r, sid)
+        assert st["hash"] == int(rep["hash"][0]) and st["flips"] == int(rep["flips"][0])
+        assert st["E"] == int(rep["E"][0]) and (st["X"] == rep["X"]).all()
+        assert (st["D"].astype(np.int64) == rep["D"]).all()
