@@ -68,7 +68,8 @@ extern "C" {
  * and SA"; reading E2). */
 #define ABS_POLICY_WINDOW 0 /* Fig. 2 / P:L305: argmin over a sliding window of l bits */
 #define ABS_POLICY_SA 1     /* Eq.(7) / Alg. 1: random bit, accepted if dE <= 0, else
-                             * with p = 2^(-dE/tau) (linear between integer exponents);
+                             * with p = exp(-dE/(k_B t)) = 2^(-dE/tau), k_B t = tau/ln 2,
+                             * as the exact Q32 integer P = floor(2^32 p) (reading E2);
                              * proposals from Philox4x32-10, key = seed, counter =
                              * (lo32(c), hi32(c), global search id, 'SAPL'), c = the
                              * search's proposal count (persists across rounds);

@@ -81,6 +81,11 @@ def lib():
         L.oracle_replay_search.argtypes = [C.c_int32, _P(C.c_int16), C.c_int32, C.c_int64, C.c_int32,
                                            _P(C.c_uint32), _P(C.c_uint32), _P(C.c_int64), _P(C.c_int64),
                                            _P(C.c_int32), _P(C.c_uint64), _P(C.c_int64), _P(C.c_uint32), _P(C.c_int64)]
+        L.oracle_replay_search_sa.restype = C.c_int
+        L.oracle_replay_search_sa.argtypes = [C.c_int32, _P(C.c_int16), C.c_int32, C.c_uint32, C.c_uint64, C.c_int64,
+                                              C.c_int32, _P(C.c_uint32), _P(C.c_uint32), _P(C.c_int64),
+                                              _P(C.c_int64), _P(C.c_int32), _P(C.c_uint64), _P(C.c_int64),
+                                              _P(C.c_uint32), _P(C.c_int64)]
         L.oracle_sa_threshold.restype = C.c_uint64
         L.oracle_sa_threshold.argtypes = [C.c_int64, C.c_int32]
         L.oracle_local_sa.restype = None
@@ -242,8 +247,10 @@ def run_lockstep(W, cfg: Config, rounds: int, want_emitted: bool = True):
     return out
 
 
-def replay_search(W, l: int, L: int, T):
-    """Rounds of one search against a given target sequence T uint32[rounds, words]."""
+def replay_search(W, l: int, L: int, T, policy: int = 0, tau: int = 1, sid: int = 0, seed: int = 1):
+    """Rounds of one search against a given target sequence T uint32[rounds, words].
+    policy 0: window of length l (Fig. 2); policy 1: SA (reading E2) at
+    temperature tau, global search id sid, Philox key seed (l unused)."""
     W = _W(W)
     n = W.shape[0]
     T = np.ascontiguousarray(np.atleast_2d(T), dtype=np.uint32)
@@ -251,14 +258,25 @@ def replay_search(W, l: int, L: int, T):
     out = dict(X=np.zeros(w, np.uint32), D=np.zeros(n, np.int64), E=np.zeros(1, np.int64),
                a=np.zeros(1, np.int32), hash=np.zeros(1, np.uint64), flips=np.zeros(1, np.int64),
                B=np.zeros((R, w), np.uint32), EB=np.zeros(R, np.int64))
-    rc = lib().oracle_replay_search(
-        n, _ptr(W, C.c_int16), int(l), int(L), R, _ptr(T, C.c_uint32),
-        _ptr(out["X"], C.c_uint32), _ptr(out["D"], C.c_int64), _ptr(out["E"], C.c_int64),
-        _ptr(out["a"], C.c_int32), _ptr(out["hash"], C.c_uint64), _ptr(out["flips"], C.c_int64),
-        _ptr(out["B"], C.c_uint32), _ptr(out["EB"], C.c_int64))
+    outs = (_ptr(out["X"], C.c_uint32), _ptr(out["D"], C.c_int64), _ptr(out["E"], C.c_int64),
+            _ptr(out["a"], C.c_int32), _ptr(out["hash"], C.c_uint64), _ptr(out["flips"], C.c_int64),
+            _ptr(out["B"], C.c_uint32), _ptr(out["EB"], C.c_int64))
+    if policy == 1:
+        rc = lib().oracle_replay_search_sa(n, _ptr(W, C.c_int16), int(tau), int(sid), int(seed) & 0xFFFFFFFFFFFFFFFF,
+                                           int(L), R, _ptr(T, C.c_uint32), *outs)
+    else:
+        rc = lib().oracle_replay_search(n, _ptr(W, C.c_int16), int(l), int(L), R, _ptr(T, C.c_uint32), *outs)
     if rc != 0:
         raise RuntimeError("oracle_replay_search rc=%d" % rc)
     return out
+
+
+def sa_tau_of(sid: int, tau_min: int, tau_max: int, levels: int) -> int:
+    """Reading E2: search sid (global id) at level j = sid mod K has
+    tau = tau_min + (tau_max - tau_min) j / (K - 1) (integer division)."""
+    K = max(1, levels)
+    j = sid % K
+    return tau_min if K == 1 else tau_min + (tau_max - tau_min) * j // (K - 1)
 
 
 # ---------------------------------------------------------------- stepwise access

@@ -102,14 +102,49 @@ __device__ __forceinline__ void philox4x32_10(uint32_t c0, uint32_t c1, uint32_t
     o[3] = c3;
 }
 
-// SA acceptance bound of an uphill move (reading E2): Eq.(7) as 2^(-dE/tau),
-// linear between integer exponents, in Q32: accept iff a uniform uint32 < it.
-__device__ __forceinline__ uint64_t sa_threshold(int dE, int tau)
+// SA acceptance (Eq.(7), reading E2): an uphill move dE > 0 is
+// accepted with p = exp(-dE/(k_B t)), k_B t = tau / ln 2, i.e. p = 2^(-dE/tau);
+// the decision is u < P for a uniform uint32 u and the Q32 integer
+// P = floor(2^32 p), computed exactly in integers:
+//   2^(-dE/tau) = 2^(-q) e^(-x),  q = dE div tau,  x = ln2 (dE mod tau) / tau,
+//   e^(-x) by its Taylor series in Q63 (terms vanish by k = 19 since x < ln 2).
+constexpr uint64_t kLn2Q64 = 0xB17217F7D1CF79ABull;  // floor(ln 2 * 2^64)
+
+__device__ __noinline__ uint64_t sa_threshold_exact(int dE, int tau)
 {
-    const int q = dE / tau;
-    const int rem = dE - q * tau;
-    if (q >= 32) return 0;
-    return ((uint64_t)1 << (32 - q)) * (uint64_t)(2 * (long long)tau - rem) / (uint64_t)(2 * (long long)tau);
+    const uint32_t ut = (uint32_t)tau;
+    const uint32_t q = (uint32_t)dE / ut;
+    const uint32_t r = (uint32_t)dE - q * ut;
+    if (q > 32) return 0;
+    // F = floor(r 2^64 / tau), Q64, by two 64/32-bit long-division steps (r < tau < 2^31)
+    const uint64_t n1 = (uint64_t)r << 32;
+    const uint64_t h = n1 / ut;
+    const uint64_t n2 = (n1 - h * ut) << 32;
+    const uint64_t F = (h << 32) | (n2 / ut);
+    const uint64_t x = __umul64hi(F, kLn2Q64);  // ln2 r / tau, Q64
+    uint64_t term = 1ull << 63, y = 1ull << 63;  // Q63
+#pragma unroll
+    for (int k = 1; k <= 20; ++k) {
+        term = __umul64hi(term, x) / (uint64_t)k;  // x^k / k!
+        y = (k & 1) ? y - term : y + term;
+    }
+    return y >> (31 + q);  // 2^32 2^(-q) y / 2^63
+}
+
+// u < P(dE, tau), deciding most draws without P: the chord C of 2^(-x) between
+// the integer exponents q and q+1 lies above the convex 2^(-x) and at most 6.2%
+// above it, so P <= C and P > 15 C / 16 - 1 (reading E2); only a
+// draw inside that band computes P.
+__device__ __forceinline__ bool sa_accept(int dE, int tau, uint32_t u)
+{
+    if (dE <= 0) return true;
+    const uint32_t q = (uint32_t)dE / (uint32_t)tau;
+    if (q > 32) return false;
+    const uint32_t r = (uint32_t)dE - q * (uint32_t)tau;
+    const long long C = (long long)(((1ull << (32 - q)) * (2ull * (uint32_t)tau - r)) / (2ull * (uint32_t)tau));
+    if ((long long)u >= C + 16) return false;
+    if ((long long)u < C - (C >> 4) - 16) return true;
+    return (uint64_t)u < sa_threshold_exact(dE, tau);
 }
 
 struct Red {
@@ -485,9 +520,16 @@ struct Round {
                                                    int sid, int n, int t, int nt, int &left, int &k, int &dk, int &xk,
                                                    int &bsz, int &cadd, int &lo_n, int &lo_s, int &lo_q)
     {
-        unsigned long long c = sm->sa_ctr + (unsigned long long)cadd;  // thread 0 wrote sa_ctr before the last barrier
-        cadd = 0;
         lo_n = 0;
+        if (left <= 0) {  // budget spent (by the early decision): only thread 0 touches sa_ctr
+            if (t == 0) sm->sa_ctr += (unsigned long long)cadd;
+            cadd = 0;
+            return false;
+        }
+        // thread 0 wrote sa_ctr before the last barrier; the batch loop below runs at least
+        // once, so its barrier orders every thread's read here before thread 0's write below
+        unsigned long long c = sm->sa_ctr + (unsigned long long)cadd;
+        cadd = 0;
         const int tau = sm->sa_tau;
         const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
         const int lane = t & 31;
@@ -539,7 +581,7 @@ struct Round {
             if (lane < nb) {
                 d = sm->sa_d[sb][lane];
                 x = sm->sa_x[sb][lane];
-                ok = d <= 0 || (uint64_t)o1 < sa_threshold(d, tau);  // Eq.(7)
+                ok = sa_accept(d, tau, o1);  // Eq.(7)
             }
             const unsigned m = __ballot_sync(kFull, ok);
             if (m) {
@@ -781,7 +823,7 @@ struct Round {
                         d = d0 + reinterpret_cast<const short *>(row)[kk] * (2 - 4 * (x0 ^ xk));
                         xn = x0;
                     }
-                    ok = d <= 0 || (uint64_t)o1 < sa_threshold(d, sm->sa_tau);  // Eq.(7)
+                    ok = sa_accept(d, sm->sa_tau, o1);  // Eq.(7)
                 }
                 const unsigned m = __ballot_sync(kFull, ok);
                 const int j = m ? __ffs(m) - 1 : -1;

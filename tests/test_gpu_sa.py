@@ -87,7 +87,7 @@ def test_sa_maxcut_ties():
 def test_sa_cold_is_descent_and_hot_accepts_all():
     n = 300
     W = random_qubo(n, 9)
-    # tau = 1: no uphill step with dE >= 32 is ever accepted (reading E2)
+    # tau = 1: no uphill step with dE >= 33 is ever accepted (P = 0, reading E2)
     s, o, gB, gEB = run_sa(W, 3, 500, 1, tmin=1, tmax=1, K=1, seed=9)
     check(s, o, gB, gEB, 3, 8)
     # huge tau: every proposal is a flip
@@ -129,3 +129,41 @@ def test_sa_degenerate_and_boundary(n, kind, tmin, tmax):
     if kind == "zeros":
         # every proposal accepted: exactly L flips per search and round after the straight phase
         assert (o["flips"] >= 3 * L).all()
+
+
+@pytest.mark.parametrize("n,S,L,steps", [
+    (300, 6, 400, 4),      # one warp x 32 bits, CTAs own their search
+    (1100, 300, 200, 2),   # one warp x 64 bits
+    (3000, 4, 600, 3),     # multi-warp (three warps)
+    (64, 6000, 60, 2),     # more searches than resident CTAs: the (search, round) queue
+])
+def test_sa_async_rounds_replay_bitexact(n, S, L, steps):
+    """Async mode with the SA policy: given the targets each search actually
+    used (trace), its trajectory is fixed by Eq.(7) and its Philox proposal
+    stream (the counter persists across rounds).  The oracle replays it:
+    every (B, E_B), the final state, flip count and trajectory hash identical."""
+    W = random_qubo(n, 20 + n)
+    tmin, tmax, K, seed = 3000, 300000, 3, 3
+    s = pkg.Solver(W, searches=S, local_flips=L, pool_size=16, seed=seed, policy=pkg.POLICY_SA,
+                   sa_tau_min=tmin, sa_tau_max=tmax, sa_levels=K, mode=pkg.MODE_ASYNC, trace=True)
+    s.search(steps)
+    tr = s.trace()
+    assert len(tr) == S * steps
+    by = {}
+    for e in tr:
+        by.setdefault(e[0], []).append(e)
+    check = range(S) if S <= 16 else list(range(0, S, 997)) + [S - 1]
+    for i in check:
+        es = sorted(by.get(i, []), key=lambda e: e[1])
+        assert [e[1] for e in es] == list(range(len(es)))
+        if not es:
+            continue
+        rep = oracle.replay_search(W, 0, L, np.array([e[2] for e in es]), policy=1,
+                                   tau=oracle.sa_tau_of(i, tmin, tmax, K), sid=i, seed=seed)
+        assert (rep["EB"] == np.array([e[4] for e in es])).all(), ("E_B", i)
+        assert all((rep["B"][r] == es[r][3]).all() for r in range(len(es))), ("B", i)
+        st = s.search_state(i)
+        assert st["hash"] == int(rep["hash"][0]) and st["flips"] == int(rep["flips"][0]), ("trajectory", i)
+        assert st["E"] == int(rep["E"][0]) and (st["X"] == rep["X"]).all()
+        assert (st["D"].astype(np.int64) == rep["D"]).all()
+    s.close()

@@ -1,7 +1,9 @@
 """Pins of the oracle's SA policy (Eq.(7) P:L116-122,
 Alg. 1, reading E2 in DESIGN.md).  None retypes the oracle's
-formulas: the threshold is held against math.exp2 and its exact integer
-points; the policy against limits whose outcome is fixed (every move
+formulas: the threshold is held against math.exp2 (within one Q32 unit),
+its exact integer points, and the exact floor decided in integer arithmetic
+(P^tau 2^dE <= 2^(32 tau) < (P+1)^tau 2^dE; nested isqrt for tau = 2^k);
+the policy against limits whose outcome is fixed (every move
 accepted / no uphill move) and against the acceptance rate a binomial
 experiment must show."""
 from __future__ import annotations
@@ -16,15 +18,15 @@ from workloads import random_qubo
 
 
 @pytest.mark.parametrize("tau", [1, 7, 1000, 2 ** 20, 2 ** 31 - 1])
-def test_threshold_integer_points_and_bounds(tau):
-    # at dE = q*tau the interpolation is exact: 2^(32-q); beyond 31 halvings it is 0
-    for q in range(0, 34):
+def test_threshold_integer_points_and_monotone(tau):
+    # at dE = q*tau, p = 2^-q exactly: 2^(32-q); below one unit (q >= 33) it is 0
+    for q in range(0, 40):
         dE = q * tau
         if dE > 2 ** 40:
             break
-        want = 2 ** (32 - q) if q < 32 else 0
+        want = 2 ** (32 - q) if q <= 32 else 0
         assert oracle.sa_threshold(dE, tau) == want
-    # monotone non-increasing, and within the linear-interpolation error of 2^-x
+    # monotone non-increasing in dE
     rng = np.random.default_rng(tau % 1000)
     prev = None
     for dE in sorted(int(v) for v in rng.integers(1, min(40 * tau, 2 ** 40), 400)):
@@ -32,9 +34,53 @@ def test_threshold_integer_points_and_bounds(tau):
         if prev is not None:
             assert P <= prev
         prev = P
-        exact = math.exp2(-dE / tau)
-        if exact > 2.0 ** -31:
-            assert abs(P / 2 ** 32 - exact) <= 0.0616 * exact + 2.0 ** -32
+
+
+def _cases(seed, count):
+    rng = np.random.default_rng(seed)
+    out = []
+    for _ in range(count):
+        tau = int(rng.choice([rng.integers(1, 50), rng.integers(1, 70000), rng.integers(1, 2 ** 31 - 1)]))
+        dE = int(rng.integers(1, min(2 ** 31 - 1, 34 * tau) + 1))
+        out.append((dE, tau))
+    return out + [(1, 2 ** 31 - 1), (2 ** 31 - 1, 2 ** 31 - 1), (2 ** 31 - 2, 2 ** 31 - 1), (2 ** 31 - 1, 1),
+                  (1, 1), (31, 1), (32, 1), (33, 1), (65, 2)]
+
+
+def test_threshold_within_one_unit_of_exp2():
+    # Eq.(7) with k_B t = tau / ln 2: P must be 2^32 * 2^(-dE/tau) to within one Q32 unit
+    for dE, tau in _cases(1, 20000):
+        q, r = divmod(dE, tau)
+        v = math.ldexp(math.exp2(-r / tau), 32 - q)   # 2^(32-q) * 2^(-r/tau), double precision
+        P = oracle.sa_threshold(dE, tau)
+        assert abs(P - v) < 1.0 + 1e-6 * max(v, 1.0) * 2 ** -20, (dE, tau, P, v)
+        if abs(v - round(v)) > 1e-4:                  # away from an integer, P is the floor
+            assert P == math.floor(v), (dE, tau, P, v)
+
+
+def test_threshold_is_exact_floor_small_tau():
+    # P = floor(2^32 2^(-dE/tau))  <=>  P^tau 2^dE <= 2^(32 tau) < (P+1)^tau 2^dE,
+    # decided in exact integer arithmetic (no floating point, no logarithm)
+    rng = np.random.default_rng(5)
+    for tau in list(range(1, 41)) + [int(v) for v in rng.integers(41, 300, 20)]:
+        for dE in sorted({1, 2, tau - 1, tau, tau + 1, 32 * tau - 1, 33 * tau - 1}
+                         | {int(v) for v in rng.integers(1, 33 * tau, 25)}):
+            if dE < 1:
+                continue
+            P = oracle.sa_threshold(dE, tau)
+            assert P ** tau * 2 ** dE <= 2 ** (32 * tau) < (P + 1) ** tau * 2 ** dE, (dE, tau, P)
+
+
+@pytest.mark.parametrize("k", [1, 2, 5, 10, 16])
+def test_threshold_is_exact_floor_power_of_two_tau(k):
+    # tau = 2^k: floor(2^(32 - dE/2^k)) = floor((2^(32*2^k - dE))^(1/2^k)) = k nested
+    # integer square roots (floor(sqrt(floor(sqrt(N)))) = floor(N^(1/4)), exactly)
+    tau = 2 ** k
+    for dE in [1, 3, tau - 1, tau + 1, 5 * tau + 7, 31 * tau + 1]:
+        v = 2 ** (32 * tau - dE)
+        for _ in range(k):
+            v = math.isqrt(v)
+        assert oracle.sa_threshold(dE, tau) == v, (dE, tau)
 
 
 def test_hot_limit_accepts_every_proposal():
@@ -77,7 +123,7 @@ def test_uphill_acceptance_rate_matches_threshold():
             down += 1
         E = s.E
     proposals_up = L - down                       # set-bit proposals are always accepted
-    p = oracle.sa_threshold(D, tau) / 2 ** 32
+    p = math.exp2(-D / tau)                       # Eq.(7) with k_B t = tau / ln 2
     sigma = math.sqrt(p * (1 - p) / proposals_up)
     assert abs(up / proposals_up - p) < 5 * sigma
 
