@@ -8,13 +8,22 @@ One step = one pass of the whole hot path over the batch of searches: the
 host GA makes one target per search, every search runs one round (straight
 search to its target + L window-policy local flips, each flip one W-row
 update evaluating n neighbours), the results are inserted into the pool
-(multi-GPU: all-gathered over NCCL first).  Inputs are synthetic (Philox
-random int16 QUBO); W (2 GiB at n = 32768) exceeds L2, so no flush
-is needed between steps.
+(multi-GPU: all-gathered over NCCL first).  Inputs are synthetic: the random
+QUBO is generated on each GPU by the library's counter-based rule
+(abs_random_qubo_dev; workloads.random_qubo_ctr is its host copy, used by the
+oracle); W (2 GiB at n = 32768) exceeds L2, so no flush is needed between
+steps.
 
-N > 1: launched by torchrun, one process per GPU; each GPU runs its own
-searches (global ids rank*S ... ) on a replicated W (weak scaling) and the
-ranks all-gather every step's results so all pools stay identical.
+--gpus N > 1: one process per GPU.  Launched by the driver under torchrun;
+run directly, bench.py re-executes itself under torch.distributed.run.  Each
+GPU runs its own searches (global ids rank*S ...) on its own replica of W
+(weak scaling) and the ranks all-gather every step's results (lockstep) or
+their elites (async), so all pools stay identical.
+
+The default line (random n = 32768, config 5) also carries `sub_results`:
+configs 2-4 (random n = 1024 with 10,000 searches, Max-Cut n = 2000, TSP
+n = 10,000), each timed for >= 2 s with its own clock record, and config 2
+in async mode for ~10 s.
 
 --impl reference: the repository's oracle (oracle/, plain C, the checker of
 the parity tests) timed on this host's cores over a bounded sample of the
@@ -24,6 +33,7 @@ from __future__ import annotations
 
 import argparse
 import json
+import math
 import multiprocessing as mp
 import os
 import statistics
@@ -39,27 +49,40 @@ if ROOT not in sys.path:
     sys.path.insert(0, ROOT)
 
 WORKLOADS = {
-    # name: (description, n, generator kwargs)
     "random32k": "random int16 QUBO n=32768 (config 5)",
     "random1k": "random int16 QUBO n=1024, 10k searches (config 2)",
     "maxcut2k": "Max-Cut G(2000, 19990) +-1 weights (config 3)",
     "tsp100": "TSP 100 cities, n=10000 one-hot (config 4)",
 }
-
+SIZES = {"random32k": 32768, "random1k": 1024, "maxcut2k": 2000, "tsp100": 10000}
+SEED = 1
 METRIC = "searched solutions/sec (n evals per flip)"
 
 
 def make_W(workload: str):
-    from workloads import maxcut_qubo, random_qubo, tsp_qubo
-    if workload == "random32k":
-        return random_qubo(32768, 1)
-    if workload == "random1k":
-        return random_qubo(1024, 1)
+    """Host copy of the workload's W (oracle, e2e input for the non-random
+    workloads, parity tests)."""
+    from workloads import maxcut_qubo, random_qubo_ctr, tsp_qubo
+    if workload in ("random32k", "random1k"):
+        return random_qubo_ctr(SIZES[workload], SEED)
     if workload == "maxcut2k":
-        return maxcut_qubo(2000, 19990, seed=1)
+        return maxcut_qubo(2000, 19990, seed=SEED)
     if workload == "tsp100":
-        return tsp_qubo(100, seed=1)
+        return tsp_qubo(100, seed=SEED)
     raise ValueError(workload)
+
+
+def make_W_device(workload: str, device: int):
+    """W in HBM: the random workloads are generated on the device (no host
+    copy per rank); the others are small and copied from the host copy."""
+    import torch
+
+    import paper_conf_icpp_yasudonitkyi20_b200 as pkg
+    if workload in ("random32k", "random1k"):
+        n = SIZES[workload]
+        Wd = torch.empty((n, n), dtype=torch.int16, device=f"cuda:{device}")
+        return pkg.random_qubo_dev(Wd, SEED)
+    return torch.from_numpy(make_W(workload)).to(f"cuda:{device}")
 
 
 # Waves of co-resident searches per step.  A lockstep step ends with its
@@ -86,17 +109,17 @@ class ClockSampler:
               "clocks_event_reasons.hw_slowdown", "clocks_event_reasons.hw_thermal_slowdown",
               "clocks_event_reasons.sw_thermal_slowdown", "power.draw"]
 
-    def __init__(self, index: int):
+    def __init__(self, index: int, period_ms: int = 100):
         self.index = index
+        self.period_ms = period_ms
         self.rows = []
-        self._stop = threading.Event()
         self._p = None
 
     def __enter__(self):
         try:
             self._p = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + ",".join(self.FIELDS),
-                 "--format=csv,noheader,nounits", "-lms", "200"], stdout=subprocess.PIPE,
+                 "--format=csv,noheader,nounits", "-lms", str(self.period_ms)], stdout=subprocess.PIPE,
                 stderr=subprocess.DEVNULL, text=True)
             self._t = threading.Thread(target=self._read, daemon=True)
             self._t.start()
@@ -136,29 +159,48 @@ _W_SHARED = None
 
 
 def _oracle_job(args):
-    l, flips, seed = args
+    """One search of the bench workload's first step, run by the oracle: the
+    GA target of round 0 (host Step 4), the round with its window
+    l and L = n (straight search + local search, Alg. 5 + Fig. 2)."""
+    sid, L = args
     import oracle
-    n = _W_SHARED.shape[0]
-    T = np.zeros((1, (n + 31) // 32), np.uint32)  # target = start: local flips only
+    W = _W_SHARED
+    n = W.shape[0]
+    cfg = oracle.Config(n=n, searches=sid + 1, local_flips=L, pool_size=64, seed=SEED)
+    T = oracle.Pool(n, 64, SEED).target(cfg, 0, sid)
+    lad = oracle.default_ladder(n)
     t = time.perf_counter()
-    out = oracle.replay_search(_W_SHARED, l, flips, T)
+    out = oracle.replay_search(W, lad[sid % len(lad)], L, T)
     return int(out["flips"][0]), time.perf_counter() - t
 
 
-def oracle_sample(W, procs: int, flips_per_proc: int):
-    """Run `procs` oracle searches in parallel (fork; W shared copy-on-write),
-    each from the zero vector with `flips_per_proc` window-policy flips.
-    Returns (flips, seconds)."""
+def oracle_sample(W, procs: int, budget_s: float):
+    """Run searches 0, 1, 2, ... of the bench workload's first step with the
+    oracle, `procs` at a time (fork; W shared copy-on-write), until about
+    `budget_s` seconds of wall time are spent.  Returns (flips, seconds,
+    searches)."""
     global _W_SHARED
     _W_SHARED = W
     import oracle
     oracle.build()
+    n = W.shape[0]
     ctx = mp.get_context("fork")
-    t = time.perf_counter()
+    flips, secs, done = 0, 0.0, 0
     with ctx.Pool(procs) as pool:
-        res = pool.map(_oracle_job, [(16, flips_per_proc, s) for s in range(procs)])
-    dt = time.perf_counter() - t
-    return sum(r[0] for r in res), dt
+        batch = procs
+        while secs < budget_s:
+            t = time.perf_counter()
+            res = pool.map(_oracle_job, [(done + i, n) for i in range(batch)])
+            dt = time.perf_counter() - t
+            flips += sum(r[0] for r in res)
+            secs += dt
+            done += batch
+            # size the next batch to the remaining budget (whole multiples of procs)
+            left = budget_s - secs
+            if left <= 0.25 * dt:
+                break
+            batch = procs * max(1, int(left / dt))
+    return flips, secs, done
 
 
 def cpu_cores() -> int:
@@ -168,12 +210,6 @@ def cpu_cores() -> int:
         return os.cpu_count() or 1
 
 
-def oracle_flips_for(n: int, seconds: float) -> int:
-    # measured oracle cost per flip ~ 35 ns * n (column walk of W) on one core
-    return max(50, int(seconds / (35e-9 * n)))
-
-
-# ------------------------------------------------------------------ arms
 def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
@@ -181,14 +217,14 @@ def run_reference(args):
     W = make_W(args.workload)
     n = W.shape[0]
     procs = min(cpu_cores(), 32)
-    flips = oracle_flips_for(n, args.ref_step_seconds)
     for _ in range(args.warmup):
-        oracle_sample(W, procs, max(50, flips // 10))
-    tot_f, tot_t = 0, 0.0
+        oracle_sample(W, procs, 0.5)
+    tot_f, tot_t, tot_s = 0, 0.0, 0
     for _ in range(args.steps):
-        f, dt = oracle_sample(W, procs, flips)
+        f, dt, s = oracle_sample(W, procs, args.ref_step_seconds)
         tot_f += f
         tot_t += dt
+        tot_s += s
     value = tot_f * n / tot_t
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": "solutions/s",
@@ -198,206 +234,326 @@ def run_reference(args):
         "config": {"workload": args.workload, "n": n, "desc": WORKLOADS[args.workload],
                    "parallelism": "host processes"},
         "cpu_baseline": {"value": value, "unit": "solutions/s", "cores": procs, "kind": "oracle",
-                         "sample": "%d oracle searches in parallel, each %d window-policy flips from X=0 per step"
-                                   % (procs, flips)},
+                         "sample": "per step: searches 0..k of the workload's first step (round-0 GA target, "
+                                   "straight search + L=n local flips each), %d at a time, ~%.0f s; %d searches "
+                                   "over %d steps" % (procs, args.ref_step_seconds, tot_s, args.steps)},
         "e2e": {"value": value, "unit": "solutions/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
     return 0
 
 
-def run_abs(args):
-    import torch
-    import torch.distributed as dist
+# ------------------------------------------------------------------ rooflines
+def _load_json(path, default=None):
+    try:
+        with open(path) as f:
+            return json.load(f)
+    except FileNotFoundError:
+        return default
 
+
+def _load_jsonl(path):
+    try:
+        with open(path) as f:
+            return [json.loads(l) for l in f if l.strip().startswith("{")]
+    except FileNotFoundError:
+        return []
+
+
+def probe_numbers():
+    """Measured denominators (bench_probe/): the random-row read bandwidth of
+    HBM (row_probe, 64 KiB rows) and of L2 (small_probe), and the int32 issue
+    rate in lanes/clk/SM (small_probe)."""
+    out = {}
+    rows = _load_jsonl(os.path.join(ROOT, "profiles", "r01_row_probe.jsonl"))
+    if rows:
+        out["hbm_row_GBps"] = max(r["GBps"] for r in rows)
+    small = _load_jsonl(os.path.join(ROOT, "profiles", "r02_small_probe.jsonl"))
+    l2 = [r for r in small if r.get("probe") == "l2_rows"]
+    for n in (1024, 2048, 10240):
+        v = [r["GBps"] for r in l2 if r["n"] == n]
+        if v:
+            out["l2_row_GBps_n%d" % n] = max(v)
+    ints = {r["op"]: r["lanes_per_clk_per_sm"] for r in small if r.get("probe") == "int32"}
+    if ints:
+        out["int32_lanes_per_clk_per_sm"] = max(ints.values())
+        out["int32_probe"] = ints
+    return out
+
+
+def roofline(workload, n, n_pad, flips, launches, kern_s, ms, local):
+    import torch
+    peaks = _load_json(os.path.join(ROOT, "MEASURED_PEAKS.json"), {}) or {}
+    hbm = float(peaks.get("hbm_gbs", 6650.0))
+    peak_src = "MEASURED_PEAKS.json hbm_gbs (copy bandwidth)" if "hbm_gbs" in peaks else \
+        "fallback 6650 GB/s (B200_PROFILING.md)"
+    probes = probe_numbers()
+    achieved = flips * 2.0 * n / kern_s / 1e9 if kern_s > 0 else None
+    roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+            "frac": (achieved / hbm) if achieved else None, "traffic": None, "traffic_unit": "GB per launch",
+            "peak_source": peak_src, "kernel": "round_kernel",
+            "algorithmic_bytes_per_launch": flips * 2.0 * n / max(1, launches),
+            "algorithmic_unit": "2n bytes (one W row) per flip",
+            "avg_launch_ms": 1e3 * kern_s / max(1, launches),
+            "kernel_share_of_step": kern_s / (ms * 1e-3) if ms > 0 else None}
+    if "hbm_row_GBps" in probes and achieved:
+        roof["row_probe_GBps"] = probes["hbm_row_GBps"]
+        roof["frac_vs_row_probe"] = achieved / probes["hbm_row_GBps"]
+    # traffic: DRAM bytes per flip of the round kernel from the committed ncu --set
+    # full capture of this workload, times this run's flips per launch
+    prof = _load_json(os.path.join(ROOT, "profiles", "round_kernel_ncu_%s.json" % workload))
+    if prof is None and workload == "random32k":
+        prof = _load_json(os.path.join(ROOT, "profiles", "round_kernel_ncu.json"))
+    if prof is not None and launches > 0:
+        if prof.get("unit") != "flips":
+            raise ValueError("ncu summary unit %r, expected 'flips'" % prof.get("unit"))
+        roof["traffic"] = prof["dram_bytes_per_unit"] * flips / launches / 1e9
+        roof["traffic_source"] = prof.get("source", "profiles/round_kernel_ncu*.json")
+        roof["traffic_over_algorithmic"] = prof["dram_bytes_per_unit"] / (2.0 * n)
+    if 2 * n_pad * n_pad <= 126 * 2 ** 20:
+        # W is L2-resident (n <= ~8k): the second roof of SURVEY 8(d) binds, n int32
+        # adds per flip against the integer pipes (measured lanes/clk/SM x SMs x max clock)
+        sms = torch.cuda.get_device_properties(local).multi_processor_count
+        mhz = float(peaks.get("sm_max_mhz", 1965.0))
+        lanes = probes.get("int32_lanes_per_clk_per_sm")
+        src = "measured (bench_probe/small_probe.cu, profiles/r02_small_probe.jsonl): %s lanes/clk/SM" % lanes
+        if lanes is None:
+            lanes = 128.0
+            src = "derived: ALU + FMA pipes, 2 x 64 int32 lanes/clk/SM (B300_MICROARCH pipe rates)"
+        int_peak = sms * lanes * mhz * 1e6 / 1e12
+        ach = flips * float(n) / kern_s / 1e12 if kern_s > 0 else None
+        l2key = "l2_row_GBps_n%d" % (1024 if n_pad <= 1024 else 2048 if n_pad <= 2048 else 10240)
+        roof.update({"bound": "alu", "achieved": ach, "peak": int_peak, "unit": "T int32 adds/s",
+                     "frac": (ach / int_peak) if ach else None,
+                     "peak_source": "%s x %d SMs x %.0f MHz (max SM clock)" % (src, sms, mhz),
+                     "row_bytes_GBps": achieved})
+        if l2key in probes and achieved:
+            roof["l2_row_probe_GBps"] = probes[l2key]
+            roof["frac_vs_l2_row_probe"] = achieved / probes[l2key]
+    return roof
+
+
+# ------------------------------------------------------------------ the GPU arm
+class Ctx:
+    def __init__(self):
+        import torch
+        import torch.distributed as dist
+        self.torch, self.dist = torch, dist
+        self.world = int(os.environ.get("WORLD_SIZE", "1"))
+        self.rank = int(os.environ.get("RANK", "0"))
+        local = int(os.environ.get("LOCAL_RANK", "0"))
+        # test hooks for exercising the multi-rank flow on a single GPU (both ranks on
+        # one device, gloo for the exchange); the driver's runs use the defaults
+        self.local = int(os.environ.get("ABS_BENCH_DEVICE", local))
+        self.backend = os.environ.get("ABS_BENCH_BACKEND", "nccl")
+        assert torch.cuda.is_available(), "bench.py needs B200 GPUs"
+        torch.cuda.set_device(self.local)
+        if self.world > 1:
+            if self.backend == "nccl":
+                dist.init_process_group("nccl", device_id=torch.device("cuda", self.local))
+            else:
+                dist.init_process_group(self.backend)
+        self.rdev = "cuda" if self.backend == "nccl" else "cpu"
+
+    def barrier(self):
+        if self.world > 1:
+            self.dist.barrier()
+
+    def allreduce(self, v, op):
+        t = self.torch.tensor([float(v)], dtype=self.torch.float64, device=self.rdev)
+        if self.world > 1:
+            self.dist.all_reduce(t, op=op)
+        return float(t.item())
+
+    def max(self, v):
+        return self.allreduce(v, self.dist.ReduceOp.MAX)
+
+    def sum(self, v):
+        return self.allreduce(v, self.dist.ReduceOp.SUM)
+
+
+def run_workload(X: Ctx, workload, steps, warmup, mode="lockstep", policy="window", searches=0, local_flips=0,
+                 min_seconds=0.0, e2e=True, W_host=None):
+    """Time `steps` steps (or, with min_seconds, enough steps to fill that
+    much time, decided after the warm-up) of one workload on every rank.
+    Returns a result dict (rank 0 fields meaningful)."""
+    torch = X.torch
     import paper_conf_icpp_yasudonitkyi20_b200 as pkg
     from paper_conf_icpp_yasudonitkyi20_b200 import dist as pdist
 
-    world = int(os.environ.get("WORLD_SIZE", "1"))
-    rank = int(os.environ.get("RANK", "0"))
-    local = int(os.environ.get("LOCAL_RANK", "0"))
-    # test hooks for exercising the multi-rank flow on a single GPU (both ranks on
-    # one device, gloo for the exchange); the driver's runs use the defaults
-    local = int(os.environ.get("ABS_BENCH_DEVICE", local))
-    backend = os.environ.get("ABS_BENCH_BACKEND", "nccl")
-    assert torch.cuda.is_available(), "bench.py needs B200 GPUs"
-    torch.cuda.set_device(local)
-    if world > 1:
-        if backend == "nccl":
-            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        else:
-            dist.init_process_group(backend)
-
-    rdev = "cuda" if backend == "nccl" else "cpu"  # device of the timing reductions
-
-    def barrier():
-        if world > 1:
-            dist.barrier()
-
-    W = make_W(args.workload)
-    n = W.shape[0]
-    S = args.searches or default_searches(args.workload, n, local)
-    L = args.local_flips or n
-    Wp = torch.from_numpy(W).pin_memory()
-    Wd = Wp.to(f"cuda:{local}", non_blocking=False)
-    mode = pkg.MODE_ASYNC if args.mode == "async" else pkg.MODE_LOCKSTEP
-    common = dict(searches=S, local_flips=L, pool_size=64, seed=1, device=local, mode=mode)
-    if args.policy == "sa":
+    n = SIZES[workload]
+    Wd = make_W_device(workload, X.local)
+    S = searches or default_searches(workload, n, X.local)
+    L = local_flips or n
+    amode = pkg.MODE_ASYNC if mode == "async" else pkg.MODE_LOCKSTEP
+    common = dict(searches=S, local_flips=L, pool_size=64, seed=SEED, device=X.local, mode=amode)
+    if policy == "sa":
         # SA policy (reading E2): a 4-level temperature ladder from the weight scale up
-        wmax = int(np.abs(W[:256].astype(np.int32)).max()) or 1  # weight scale from a row sample
+        wmax = int(Wd[:256].abs().max().item()) or 1  # weight scale from a row sample
         common.update(policy=pkg.POLICY_SA, sa_tau_min=max(1, wmax // 4), sa_tau_max=8 * wmax, sa_levels=4)
-    solver = pkg.Solver(Wd, search_offset=rank * S, external_merge=(world > 1 and mode == pkg.MODE_LOCKSTEP),
-                        **common)
-    del Wd
+    ext = X.world > 1 and amode == pkg.MODE_LOCKSTEP
+    solver = pkg.Solver(Wd, search_offset=X.rank * S, external_merge=ext, **common)
 
     def step(s):
-        if world > 1:
+        if X.world > 1:
             pdist.lockstep_step(s)
         else:
             s.search(1)
 
     def run_steps(s, k):
-        if mode == pkg.MODE_ASYNC:
+        if amode == pkg.MODE_ASYNC:
             # one persistent launch for all k rounds of every search (P:L426: the
             # blocks run asynchronously); ranks then all-gather their elites
             s.search(k)
-            if world > 1:
+            if X.world > 1:
                 pdist.exchange_elites(s, 64)
         else:
             for _ in range(k):
                 step(s)
 
-    run_steps(solver, args.warmup)
-    barrier()
+    X.barrier()
     torch.cuda.synchronize()
+    tw = time.perf_counter()
+    run_steps(solver, warmup)
+    torch.cuda.synchronize()
+    warm_s = time.perf_counter() - tw
+    if min_seconds > 0:
+        per = warm_s / max(1, warmup)
+        if amode == pkg.MODE_ASYNC:
+            # one launch per call: calibrate on a longer (untimed) call than the warm-up
+            k = max(1, int(0.15 * min_seconds / max(per, 1e-6)))
+            torch.cuda.synchronize()
+            tw = time.perf_counter()
+            run_steps(solver, k)
+            torch.cuda.synchronize()
+            per = (time.perf_counter() - tw) / k
+        steps = int(X.max(max(steps, math.ceil(min_seconds / max(per, 1e-6)))))
     st0 = solver.stats()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local) as clk:
-        barrier()
+    with ClockSampler(X.local) as clk:
+        X.barrier()
         torch.cuda.synchronize()
         ev0.record()
-        run_steps(solver, args.steps)
+        run_steps(solver, steps)
         ev1.record()
         torch.cuda.synchronize()
-        barrier()
+        X.barrier()
     st1 = solver.stats()
     ms = ev0.elapsed_time(ev1)
     flips = st1["flips"] - st0["flips"]
     kern_s = st1["search_seconds"] - st0["search_seconds"]
     launches = st1["round_kernel_launches"] - st0["round_kernel_launches"]
     all_launches = st1["kernel_launches"] - st0["kernel_launches"]
-    t_ms = torch.tensor([ms], dtype=torch.float64, device=rdev)
-    t_fl = torch.tensor([flips], dtype=torch.float64, device=rdev)
-    if world > 1:
-        dist.all_reduce(t_ms, op=dist.ReduceOp.MAX)
-        dist.all_reduce(t_fl, op=dist.ReduceOp.SUM)
-    ms_max = float(t_ms.item())
-    flips_all = float(t_fl.item())
-    value = flips_all * n / (ms_max * 1e-3)
-
-    # roofline of the dominant kernel (the round kernel): algorithmic bytes =
-    # one W row (2n bytes) per flip; time = its CUDA-event duration.
-    peaks = {}
-    try:
-        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
-    except Exception:
-        pass
-    hbm = float(peaks.get("hbm_gbs", 6650.0))
-    peak_src = "measured" if "hbm_gbs" in peaks else "fallback"
-    achieved = flips * 2.0 * n / kern_s / 1e9 if kern_s > 0 else None
-    # traffic: DRAM bytes per flip of the round kernel from the committed ncu
-    # --set full capture (profiles/round_kernel_ncu.json), times this run's flips
-    # per launch; only for the workload it was captured on.
-    traffic = None
-    try:
-        prof = json.load(open(os.path.join(ROOT, "profiles", "round_kernel_ncu.json")))
-        if args.workload == "random32k" and launches > 0:
-            traffic = prof["dram_bytes_per_flip"] * flips / launches / 1e9
-    except Exception:
-        pass
-    roof = {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-            "frac": (achieved / hbm) if achieved else None, "traffic": traffic, "traffic_unit": "GB per launch",
-            "peak_source": peak_src, "kernel": "round_kernel",
-            "algorithmic_bytes_per_launch": flips * 2.0 * n / max(1, launches),
-            "avg_launch_ms": 1e3 * kern_s / max(1, launches),
-            "kernel_share_of_step": kern_s / (ms * 1e-3) if ms > 0 else None}
-    n_pad = int(st1["n_pad"])
-    if 2 * n_pad * n_pad <= 126 * 2 ** 20:
-        # W is L2-resident (n <= ~8k): the second roof of SURVEY §8(d) binds, n int32
-        # adds per flip against the INT32 pipe: 64 lanes/clk/SM (IMAD/IADD3 issue
-        # every 2 cycles per SMSP, B300_MICROARCH "pipe rates") x SMs x max SM clock
-        sms = torch.cuda.get_device_properties(local).multi_processor_count
-        mhz = float(peaks.get("sm_max_mhz", 1965.0))
-        int_peak = sms * 64 * mhz * 1e6 / 1e12
-        ach = flips * float(n) / kern_s / 1e12 if kern_s > 0 else None
-        roof.update({"bound": "alu", "achieved": ach, "peak": int_peak, "unit": "T int32 adds/s",
-                     "frac": (ach / int_peak) if ach else None,
-                     "peak_source": "derived: %d SMs x 64 int32 lanes/clk x %.0f MHz" % (sms, mhz),
-                     "row_bytes_GBps": achieved})
+    ms_max = X.max(ms)
+    flips_all = X.sum(flips)
+    res = {
+        "value": flips_all * n / (ms_max * 1e-3), "unit": "solutions/s", "steps": steps, "warmup": warmup,
+        "ms_per_step": ms_max / steps, "seconds": ms_max * 1e-3, "flips_per_step": flips_all / steps,
+        "gpu_launches": int(all_launches),
+        "config": {"workload": workload, "desc": WORKLOADS[workload], "n": n, "searches_per_gpu": S,
+                   "local_flips": L, "pool": 64, "mode": mode, "policy": policy,
+                   "w_source": "generated on device (abs_random_qubo_dev)" if workload.startswith("random")
+                   else "host generator, copied once"},
+        "roofline": roofline(workload, n, int(st1["n_pad"]), flips, launches, kern_s, ms, X.local),
+        "clocks": clk.summary(),
+    }
     solver.close()
     del solver
     torch.cuda.synchronize()
 
-    # ---------------- end to end through the public API with host buffers
-    e2e = None
-    if not args.no_e2e:
-        barrier()
+    if e2e:
+        # end to end through the public API with HOST buffers: abs_create from pinned host
+        # W (H2D inside the timed region), the steps, abs_best (D2H of the result)
+        if W_host is None:
+            W_host = torch.empty(Wd.shape, dtype=torch.int16, pin_memory=True)
+            W_host.copy_(Wd)  # staging of the input, outside the timed region
+        Wh = W_host.numpy()
+        del Wd
         torch.cuda.synchronize()
+        X.barrier()
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
-        s2 = pkg.Solver(Wp.numpy(), search_offset=rank * S,
-                        external_merge=(world > 1 and mode == pkg.MODE_LOCKSTEP), **common)
-        run_steps(s2, args.steps)
-        Xb, Eb = s2.best() if world == 1 else (None, None)
+        s2 = pkg.Solver(Wh, search_offset=X.rank * S, external_merge=ext, **common)
+        run_steps(s2, steps)
+        Xb, Eb = s2.best() if X.world == 1 else (None, None)
         e1.record()
         torch.cuda.synchronize()
         st2 = s2.stats()
         s2.close()
-        ems = e0.elapsed_time(e1)
-        t2 = torch.tensor([ems], dtype=torch.float64, device=rdev)
-        f2 = torch.tensor([st2["flips"]], dtype=torch.float64, device=rdev)
-        if world > 1:
-            dist.all_reduce(t2, op=dist.ReduceOp.MAX)
-            dist.all_reduce(f2, op=dist.ReduceOp.SUM)
-        e2e = {"value": float(f2.item()) * n / (float(t2.item()) * 1e-3), "unit": "solutions/s",
-               "h2d_bytes_per_step": st2["h2d_bytes"] / args.steps,
-               "d2h_bytes_per_step": (st2["d2h_bytes"] + 8 * ((n + 31) // 32)) / args.steps,
-               "includes": "abs_create from pinned host W (H2D 2n^2 bytes) + steps + abs_best"}
+        ems = X.max(e0.elapsed_time(e1))
+        f2 = X.sum(st2["flips"])
+        res["e2e"] = {"value": f2 * n / (ems * 1e-3), "unit": "solutions/s",
+                      "h2d_bytes_per_step": st2["h2d_bytes"] / steps,
+                      "d2h_bytes_per_step": (st2["d2h_bytes"] + 8 * ((n + 31) // 32)) / steps,
+                      "includes": "abs_create from pinned host W (H2D 2n^2 bytes) + steps + abs_best"}
+    return res
+
+
+def run_abs(args):
+    X = Ctx()
+    main = run_workload(X, args.workload, args.steps, args.warmup, mode=args.mode, policy=args.policy,
+                        searches=args.searches, local_flips=args.local_flips, e2e=not args.no_e2e)
+    n = SIZES[args.workload]
+
+    subs = {}
+    if not args.no_sub and args.workload == "random32k" and args.mode == "lockstep" and args.policy == "window":
+        # configs 2-4 of BASELINE.json, each >= 2 s, and config 2 async for ~10 s (SURVEY 8(d))
+        for w in ("random1k", "maxcut2k", "tsp100"):
+            r = run_workload(X, w, 3, 3, min_seconds=args.sub_seconds, e2e=False)
+            subs[w] = {k: r[k] for k in ("value", "unit", "steps", "ms_per_step", "seconds", "roofline", "clocks",
+                                         "config", "gpu_launches")}
+        r = run_workload(X, "random1k", 3, 3, mode="async", min_seconds=args.async_seconds, e2e=False)
+        subs["random1k_async"] = {k: r[k] for k in ("value", "unit", "steps", "seconds", "roofline", "clocks",
+                                                    "config", "gpu_launches")}
+        subs["random1k_async"]["note"] = "config 2: throughput of one asynchronous abs_search call of ~%.0f s " \
+                                         "(persistent kernel + host GA thread, Fig. 5)" % args.async_seconds
 
     # ---------------- cpu baseline (oracle), rank 0 at N = 1 only
     cpu = None
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+    if X.rank == 0 and X.world == 1 and not args.no_cpu_baseline:
+        W = make_W(args.workload)
         procs = min(cpu_cores(), 32)
-        fl = oracle_flips_for(n, args.cpu_seconds)
-        f, dt = oracle_sample(W, procs, fl)
+        f, dt, s = oracle_sample(W, procs, args.cpu_seconds)
         cpu = {"value": f * n / dt, "unit": "solutions/s", "cores": procs, "kind": "oracle",
-               "sample": "%d oracle searches in parallel, %d window-policy flips each from X=0 (%.1f s)"
-                         % (procs, fl, dt)}
+               "sample": "searches 0..%d of the bench step (round-0 GA targets, straight search + L=n local "
+                         "flips each), %d at a time on %d cores, %.1f s" % (s - 1, procs, procs, dt)}
 
-    if rank == 0:
+    if X.rank == 0:
         line = {
-            "metric": METRIC, "value": value, "unit": "solutions/s", "n_gpus": world,
-            "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms_max / args.steps,
+            "metric": METRIC, "value": main["value"], "unit": "solutions/s", "n_gpus": X.world,
+            "steps": main["steps"], "warmup": args.warmup, "ms_per_step": main["ms_per_step"],
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int32",
-            "data": "synthetic (Philox random int16 QUBO, P:L468)" if args.workload.startswith("random")
-            else "synthetic",
-            "config": {"workload": args.workload, "desc": WORKLOADS[args.workload], "n": n,
-                       "searches_per_gpu": S, "local_flips": L, "pool": 64, "mode": args.mode, "policy": args.policy,
-                       "parallelism": "dp%d (replicated W, independent searches)" % world,
-                       "l2": "inputs larger than L2 (W = %d MiB)" % (2 * n * n >> 20)
-                       if 2 * n * n > 126 * 2 ** 20 else "W fits in L2 (resident by design)"},
-            "flips_per_step": flips_all / args.steps,
-            "roofline": roof,
+            "data": "synthetic (Philox random int16 QUBO generated on device, P:L468)"
+            if args.workload.startswith("random") else "synthetic",
+            "config": dict(main["config"], parallelism="dp%d (replicated W, independent searches)" % X.world,
+                           l2="inputs larger than L2 (W = %d MiB)" % (2 * n * n >> 20)
+                           if 2 * n * n > 126 * 2 ** 20 else "W fits in L2 (resident by design)"),
+            "flips_per_step": main["flips_per_step"],
+            "roofline": main["roofline"],
             "cpu_baseline": cpu,
-            "e2e": e2e,
-            "gpu_launches": int(all_launches),
-            "clocks": clk.summary(),
+            "e2e": main.get("e2e"),
+            "gpu_launches": main["gpu_launches"],
+            "clocks": main["clocks"],
+            "sub_results": subs or None,
             "paper_context": "1.24e12 solutions/s on 4x RTX 2080 Ti at n=1024; 4.39e11 at n=32768 (P:L529, P:L544)",
         }
         print(json.dumps(line), flush=True)
-    if world > 1:
-        dist.destroy_process_group()
+    if X.world > 1:
+        X.dist.destroy_process_group()
     return 0
+
+
+def relaunch_distributed(n: int) -> int:
+    """bench.py --gpus N run directly: re-execute under torch.distributed.run,
+    one process per GPU (the driver's own launch form)."""
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(n),
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
 
 
 def main():
@@ -413,11 +569,20 @@ def main():
     ap.add_argument("--local-flips", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-sub", action="store_true", help="skip the configs 2-4 sub-results")
+    ap.add_argument("--sub-seconds", type=float, default=2.5)
+    ap.add_argument("--async-seconds", type=float, default=10.0)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-step-seconds", type=float, default=8.0)
     args = ap.parse_args()
     if args.warmup < 3:
         print("warning: --warmup < 3 violates the timing rules", file=sys.stderr)
+    world = os.environ.get("WORLD_SIZE")
+    if world is None and args.gpus > 1:
+        return relaunch_distributed(args.gpus)
+    if world is not None and int(world) != args.gpus:
+        print("bench.py: --gpus %d but WORLD_SIZE=%s (one process per GPU)" % (args.gpus, world), file=sys.stderr)
+        return 2
     if args.impl == "reference":
         return run_reference(args)
     return run_abs(args)

@@ -46,6 +46,10 @@ extern "C" {
 #define ABS_EINVAL (-1)   /* bad argument (n out of range, W not symmetric, NULL, ...) */
 #define ABS_ENOMEM (-2)   /* host or device allocation failed */
 #define ABS_ECUDA (-3)    /* CUDA runtime error or no sm_100 device */
+#define ABS_ENCCL (-4)    /* reserved for the multi-GPU elite exchange; the
+                           * library itself makes no NCCL call: the exchange runs in the
+                           * caller's process group (dist.py, torch.distributed over NCCL),
+                           * which reports its own errors */
 #define ABS_ESTATE (-5)   /* call not valid in the current state */
 #define ABS_EEMPTY (-6)   /* no finite-energy solution in the pool yet */
 #define ABS_ERANGE (-7)   /* a Delta left the int32 range (cannot happen for n <= 32768) */
@@ -77,7 +81,8 @@ extern "C" {
                              * local_flips counts proposals. */
 
 typedef struct abs_config {
-    int32_t searches;       /* searches run by this context (per GPU); 0 -> 148 */
+    int32_t searches;       /* searches run by this context (per GPU); 0 -> one wave:
+                             * abs_device_searches(n, device) (148 at n = 32768) */
     int32_t search_offset;  /* global id of this context's first search
                              * (multi-GPU partitioning) */
     int64_t local_flips;    /* L: forced flips of the local search per round
@@ -169,10 +174,14 @@ ABS_API int abs_seed_pool(abs_ctx *c, const uint32_t *X, int32_t count);
  *     otherwise every search does exactly `steps` rounds. */
 ABS_API int abs_search(abs_ctx *c, int64_t steps);
 
-/* Best pool entry (pool[0]): X_out host (words(n) words), *E_out host.
- * ABS_EEMPTY if no finite energy exists yet. */
+/* Best solution found so far: the host keeps the pool sorted by energy,
+ * E(X_0) < E(X_1) < ..., so this is pool[0].  X_out: host,
+ * words(n) words; *E_out: host.  ABS_EEMPTY if no finite energy exists yet. */
 ABS_API int abs_best(const abs_ctx *c, uint32_t *X_out, int64_t *E_out);
 
+/* Counters since create (abs_stats above): flips, and searched solutions =
+ * flips * n, the paper's search-rate accounting (every flip evaluates all n
+ * neighbours in O(1) each); device seconds by CUDA events. */
 ABS_API int abs_stats_get(const abs_ctx *c, abs_stats *s);
 
 /* Top-k finite pool entries (ascending energy).  X_out: k*words(n) words,
@@ -233,6 +242,8 @@ ABS_API int abs_trace_get(const abs_ctx *c, int64_t i, int32_t *s_out, int32_t *
 ABS_API int abs_search_state(const abs_ctx *c, int32_t s, uint32_t *X_out, int32_t *delta_out, int64_t *E_out,
                      int32_t *a_out, int32_t *l_out, uint64_t *hash_out, int64_t *flips_out);
 
+/* Stops the host GA thread (the host side of the system),
+ * frees the context's device and pinned host memory.  c may be NULL. */
 ABS_API void abs_destroy(abs_ctx *c);
 
 ABS_API const char *abs_strerror(int rc);
@@ -270,6 +281,18 @@ ABS_API int abs_qubo_to_ising(int32_t n, const int16_t *W, int32_t *J2_out, int3
  * count that fills the GPU in one wave ("blocks ... run in
  * parallel").  Needs a visible CUDA device (ABS_ECUDA otherwise). */
 ABS_API int abs_device_searches(int32_t n, int32_t device, int32_t *out);
+
+/* Synthetic random QUBO instance (the paper's random benchmark, P:L468:
+ * "uniform random" weights) generated directly in device memory, so each
+ * rank of a multi-GPU run builds its replica of W (2 GiB at n = 32768)
+ * without staging it through host memory.  W_dev: n*n int16,
+ * row-major, device memory of `device` (-1: current), owned by the caller;
+ * overwritten with a symmetric W whose upper triangle (i <= j) is
+ *   W_ij = int16 half (j & 1) of word ((j >> 1) & 3) of
+ *          Philox4x32-10(key = (lo32 seed, hi32 seed), counter = (i, j >> 3, 0x52514243, 0))
+ * (i.i.d. uniform over all 65536 values) and W_ji = W_ij.  Blocking.
+ * ABS_EINVAL for n outside [1, 32768] or W_dev == NULL, ABS_ECUDA on a CUDA error. */
+ABS_API int abs_random_qubo_dev(int32_t n, uint64_t seed, int16_t *W_dev, int32_t device);
 
 /* Library version string. */
 ABS_API const char *abs_version(void);

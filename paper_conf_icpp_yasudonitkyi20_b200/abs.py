@@ -81,6 +81,7 @@ EXPORTS = [
     "abs_config_init", "abs_create", "abs_create_dev", "abs_seed_pool", "abs_search", "abs_best",
     "abs_stats_get", "abs_pool_get", "abs_pool_insert", "abs_energy", "abs_energy_dev", "abs_round_results",
     "abs_round_targets", "abs_trace_count", "abs_trace_get", "abs_search_state", "abs_debug_timing", "abs_destroy", "abs_strerror", "abs_last_error", "abs_device_searches", "abs_ising_to_qubo", "abs_qubo_to_ising", "abs_version",
+    "abs_random_qubo_dev",
 ]
 
 _lib = None
@@ -138,6 +139,8 @@ def load(build_if_missing: bool = True):
     if hasattr(L, "abs_ising_to_qubo") or not os.environ.get("ABS_LIB"):
         L.abs_ising_to_qubo.argtypes = [C.c_int32, vp, vp, vp, P(C.c_int64)]
         L.abs_qubo_to_ising.argtypes = [C.c_int32, vp, vp, vp, P(C.c_int64)]
+    if hasattr(L, "abs_random_qubo_dev") or not os.environ.get("ABS_LIB"):
+        L.abs_random_qubo_dev.argtypes = [C.c_int32, C.c_uint64, vp, C.c_int32]
     L.abs_version.argtypes = []
     L.abs_version.restype = C.c_char_p
     for name in EXPORTS:
@@ -384,6 +387,16 @@ def device_searches(n: int, device: int = 0) -> int:
     out = C.c_int32()
     _check(load().abs_device_searches(int(n), int(device), C.byref(out)), "abs_device_searches")
     return int(out.value)
+
+
+def random_qubo_dev(W, seed: int = 1):
+    """Fill the CUDA int16 tensor W [n, n] with the synthetic random QUBO of
+    abs_random_qubo_dev, generated on W's device."""
+    assert W.is_cuda and str(W.dtype) == "torch.int16" and W.dim() == 2 and W.shape[0] == W.shape[1]
+    assert W.is_contiguous()
+    _check(load().abs_random_qubo_dev(int(W.shape[0]), C.c_uint64(int(seed) & 0xFFFFFFFFFFFFFFFF),
+                                      C.c_void_p(W.data_ptr()), int(W.device.index)), "abs_random_qubo_dev")
+    return W
 
 
 def version() -> str:

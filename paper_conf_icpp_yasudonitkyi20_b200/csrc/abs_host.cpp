@@ -284,7 +284,6 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
     abs_config cfg;
     abs_config_init(&cfg);
     if (cfg_in) cfg = *cfg_in;
-    if (cfg.searches == 0) cfg.searches = 148;
     if (cfg.searches < 0 || cfg.search_offset < 0) return fail(ABS_EINVAL, "bad searches/search_offset");
     if (cfg.local_flips == 0) cfg.local_flips = n;  // reading C8
     if (cfg.local_flips < 0 || cfg.local_flips > INT32_MAX) return fail(ABS_EINVAL, "bad local_flips");
@@ -322,6 +321,11 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
     ABS_CU(cudaGetDeviceProperties(&prop, dev));
     if (prop.major != 10) return fail(ABS_ECUDA, "libabs is built for sm_100a (B200); device is sm_" +
                                                      std::to_string(prop.major) + std::to_string(prop.minor));
+    if (cfg.searches == 0) {  // one wave: every SM filled with co-resident searches
+        int32_t one_wave = 0;
+        ABS_CK(abs_device_searches(n, dev, &one_wave));
+        cfg.searches = one_wave;
+    }
 
     abs_ctx *c = new (std::nothrow) abs_ctx();
     if (!c) return fail(ABS_ENOMEM, "host allocation");
@@ -1063,6 +1067,7 @@ const char *abs_strerror(int rc)
     case ABS_EINVAL: return "invalid argument";
     case ABS_ENOMEM: return "out of memory";
     case ABS_ECUDA: return "CUDA error";
+    case ABS_ENCCL: return "NCCL error (multi-GPU exchange)";
     case ABS_ESTATE: return "invalid state";
     case ABS_EEMPTY: return "pool has no finite-energy solution";
     case ABS_ERANGE: return "delta out of int32 range";
@@ -1136,6 +1141,19 @@ int abs_device_searches(int32_t n, int32_t device, int32_t *out)
     ABS_CK(rc);
     ABS_CU(e2);
     *out = per_sm * sms;
+    return ABS_OK;
+}
+
+int abs_random_qubo_dev(int32_t n, uint64_t seed, int16_t *W_dev, int32_t device)
+{
+    if (n < 1 || n > ABS_N_MAX || !W_dev) return fail(ABS_EINVAL, "abs_random_qubo_dev: n out of range or W_dev == NULL");
+    int prev = 0;
+    ABS_CU(cudaGetDevice(&prev));
+    if (device >= 0) ABS_CU(cudaSetDevice(device));
+    int rc = launch_random_qubo(W_dev, n, seed, 0);
+    if (rc == 0) rc = (int)cudaDeviceSynchronize();
+    cudaSetDevice(prev);
+    ABS_CU((cudaError_t)rc);
     return ABS_OK;
 }
 

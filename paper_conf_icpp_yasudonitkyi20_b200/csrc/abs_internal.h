@@ -1,5 +1,6 @@
 // Internal declarations shared by the host library (abs_host.cpp) and the
-// sm_100a kernels (abs_kernels.cu).  Not part of the ABI.
+// sm_100a kernels (abs_round.cu, abs_setup.cu, abs_init_mma.cu).  Not part of
+// the ABI.
 #pragma once
 #include <cstddef>
 #include <cstdint>
@@ -102,6 +103,8 @@ struct AsyncArgs {
 int launch_prepare_w(const int16_t *W_in, int32_t n, int32_t n_pad, int16_t *Wz, int32_t *diag,
                      unsigned long long *asym_count, cudaStream_t st);
 int launch_rowmax(const Instance &I, cudaStream_t st);
+// synthetic random QUBO n x n (row-major, dense) into W (abs_random_qubo_dev)
+int launch_random_qubo(int16_t *W, int32_t n, uint64_t seed, cudaStream_t st);
 int launch_zero_start(const Instance &I, SearchState &S, int32_t s0, int32_t s1, cudaStream_t st);
 // q == nullptr: lockstep round (one CTA per search); otherwise the persistent
 // asynchronous kernel (grid = min(S, resident CTAs), *grid_out).

@@ -157,6 +157,71 @@ __global__ void __launch_bounds__(kInitT) batch_init_kernel(const int16_t *__res
     }
 }
 
+
+// ------------------------------------------------------------------ synthetic instance
+// Synthetic random QUBO ("uniform random" weights), generated on the
+// device so that every rank of a multi-GPU run builds its replica of W in HBM
+// (2 GiB at n = 32768) without host memory.  W is symmetric; the upper
+// triangle (i <= j) is i.i.d. uniform over all int16:
+//   W_ij = int16 half (j & 1) of word ((j >> 1) & 3) of
+//          Philox4x32-10(key = seed, counter = (i, j >> 3, 'RQBC', 0)),
+// and W_ji = W_ij.  (workloads.random_qubo_ctr is the host copy of this rule.)
+constexpr uint32_t kTagRqbc = 0x52514243u;  // 'RQBC'
+
+// Philox4x32-10 (Salmon et al., SC'11) in place on a counter block
+__device__ __forceinline__ void philox4x32_10(uint32_t (&c)[4], uint32_t k0, uint32_t k1)
+{
+#pragma unroll
+    for (int r = 0; r < 10; ++r) {
+        const uint32_t hi0 = __umulhi(0xD2511F53u, c[0]), lo0 = 0xD2511F53u * c[0];
+        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c[2]), lo1 = 0xCD9E8D57u * c[2];
+        const uint32_t n0 = hi1 ^ c[1] ^ k0, n2 = hi0 ^ c[3] ^ k1;
+        c[0] = n0;
+        c[1] = lo1;
+        c[2] = n2;
+        c[3] = lo0;
+        k0 += 0x9E3779B9u;
+        k1 += 0xBB67AE85u;
+    }
+}
+constexpr int kGenTile = 64;
+
+// One 64 x 64 tile (I, J), I <= J, per CTA (256 threads): the upper values of
+// the tile go through shared memory, so the mirror tile (J, I) is written with
+// coalesced rows too.
+__global__ void __launch_bounds__(256) random_qubo_kernel(int16_t *__restrict__ W, int n, uint64_t seed,
+                                                          int tiles)
+{
+    __shared__ int16_t S[kGenTile][kGenTile + 2];
+    // tile pair from the linear index over the upper triangle of tiles (row-major)
+    int I = 0, rem = (int)blockIdx.x;
+    while (rem >= tiles - I) {
+        rem -= tiles - I;
+        ++I;
+    }
+    const int J = I + rem;
+    const int i0 = I * kGenTile, j0 = J * kGenTile;
+    for (int c = threadIdx.x; c < kGenTile * (kGenTile / 8); c += blockDim.x) {
+        const int r = c >> 3, g = c & 7;  // row r of the tile, column group g (8 columns)
+        uint32_t o[4] = {(uint32_t)(i0 + r), (uint32_t)((j0 >> 3) + g), kTagRqbc, 0u};
+        philox4x32_10(o, (uint32_t)seed, (uint32_t)(seed >> 32));
+#pragma unroll
+        for (int e = 0; e < 8; ++e) S[r][8 * g + e] = (int16_t)(uint16_t)(o[e >> 1] >> (16 * (e & 1)));
+    }
+    __syncthreads();
+    for (int c = threadIdx.x; c < kGenTile * kGenTile; c += blockDim.x) {
+        const int r = c / kGenTile, q = c % kGenTile;
+        {  // tile (I, J): row i0 + r; on the diagonal tile, below the diagonal the mirrored value
+            const int i = i0 + r, j = j0 + q;
+            if (i < n && j < n) W[(size_t)i * n + j] = (I == J && q < r) ? S[q][r] : S[r][q];
+        }
+        if (I != J) {  // mirror tile (J, I): row j0 + r holds W_{j0+r, i0+q} = S[q][r]
+            const int i = j0 + r, j = i0 + q;
+            if (i < n && j < n) W[(size_t)i * n + j] = S[q][r];
+        }
+    }
+}
+
 }  // namespace
 
 
@@ -192,6 +257,15 @@ int launch_batch_init(const Instance &I, const uint8_t *X, int32_t row_bytes, in
     const size_t smem = (size_t)kInitB * (I.n_pad / 32) * sizeof(uint32_t);
     cudaFuncSetAttribute(batch_init_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     batch_init_kernel<<<grid, kInitT, smem, st>>>(I.Wz, I.diag, I.n, I.n_pad, X, row_bytes, count, E, delta);
+    return (int)cudaGetLastError();
+}
+
+
+int launch_random_qubo(int16_t *W, int32_t n, uint64_t seed, cudaStream_t st)
+{
+    const int tiles = (n + kGenTile - 1) / kGenTile;
+    const int pairs = tiles * (tiles + 1) / 2;
+    random_qubo_kernel<<<pairs, 256, 0, st>>>(W, n, seed, tiles);
     return (int)cudaGetLastError();
 }
 

@@ -283,10 +283,10 @@ def test_bench_configuration_sampled(workload):
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import bench
 
-    W = bench.make_W(workload)
+    W = bench.make_W(workload)                 # host copy (oracle)
     n = W.shape[0]
     S = bench.default_searches(workload, n, 0)
-    s = make(W, searches=S, local_flips=n, pool_size=64, seed=1)
+    s = make(bench.make_W_device(workload, 0), searches=S, local_flips=n, pool_size=64, seed=1)  # as bench.py
     s.search(1)
     B, EB = s.round_results()
     cfg = ocfg(n, S, n, 64, 1)
@@ -455,10 +455,10 @@ def test_full_size_bench_three_rounds_replay():
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import bench
 
-    W = bench.make_W("random32k")
+    W = bench.make_W("random32k")              # host copy (oracle)
     n = W.shape[0]
     S = bench.default_searches("random32k", n, 0)
-    s = make(W, searches=S, local_flips=n, pool_size=64, seed=1)
+    s = make(bench.make_W_device("random32k", 0), searches=S, local_flips=n, pool_size=64, seed=1)
     Ts, Bs, EBs = [], [], []
     for _ in range(3):
         s.search(1)
@@ -496,3 +496,24 @@ def test_full_size_bench_three_rounds_replay():
         assert st["hash"] == int(rep["hash"][0]) and st["flips"] == int(rep["flips"][0])
         assert st["E"] == int(rep["E"][0]) and (st["X"] == rep["X"]).all()
         assert (st["D"].astype(np.int64) == rep["D"]).all()
+
+
+# ---------------------------------------------------------------- synthetic instance on the device (a1)
+@pytest.mark.parametrize("n", [1, 7, 8, 63, 64, 65, 1000, 4097])
+def test_random_qubo_dev_equals_host_generator(n):
+    from workloads import random_qubo_ctr
+    Wd = torch.empty((n, n), dtype=torch.int16, device="cuda:0")
+    abs_b200.random_qubo_dev(Wd, 77)
+    assert (Wd.cpu().numpy() == random_qubo_ctr(n, 77)).all()
+
+
+def test_random_qubo_dev_full_size_rows():
+    from workloads import random_qubo_ctr_rows
+    n = 32768
+    Wd = torch.empty((n, n), dtype=torch.int16, device="cuda:0")
+    abs_b200.random_qubo_dev(Wd, 1)
+    for r0 in (0, 4093, 16000, 32765):
+        assert (Wd[r0:r0 + 3].cpu().numpy() == random_qubo_ctr_rows(n, 1, r0, r0 + 3)).all(), r0
+    # symmetric (columns = rows) on a sample
+    for c in (0, 12345, 32767):
+        assert (Wd[:, c].cpu() == Wd[c].cpu()).all()

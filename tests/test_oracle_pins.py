@@ -413,3 +413,22 @@ def test_replay_matches_lockstep_search():
     assert (rep["X"] == full["X"][0]).all() and rep["E"][0] == full["E"][0]
     assert rep["hash"][0] == full["hash"][0] and rep["flips"][0] == full["flips"][0]
     assert (rep["EB"] == full["EB"][:, 0]).all()
+
+
+def test_counter_based_random_qubo_generator():
+    """workloads.random_qubo_ctr (the host copy of abs_random_qubo_dev): every
+    entry follows the stated Philox rule, checked with the ORACLE's Philox
+    (pinned by the Random123 vectors) on a sample; symmetric; uniform moments
+    (mean -1/2, sd 65536/sqrt(12)); the row-range form equals the full matrix."""
+    from workloads import random_qubo_ctr, random_qubo_ctr_rows
+    n, seed = 1500, (7 << 32) | 3
+    W = random_qubo_ctr(n, seed)
+    assert (W == W.T).all()
+    rng = np.random.default_rng(0)
+    for i, j in [(0, 0), (0, n - 1), (n - 1, n - 1)] + [tuple(sorted(v)) for v in rng.integers(0, n, (40, 2))]:
+        o = oracle.philox4x32_10([i, j >> 3, 0x52514243, 0], [seed & 0xFFFFFFFF, seed >> 32])
+        v = (int(o[(j >> 1) & 3]) >> (16 * (j & 1))) & 0xFFFF
+        assert int(W[i, j]) == (v - 65536 if v >= 32768 else v)
+    assert (random_qubo_ctr_rows(n, seed, 700, 710) == W[700:710]).all()
+    big = random_qubo_ctr(4096, 1).astype(np.float64)
+    assert abs(big.mean() + 0.5) < 60 and abs(big.std() - 65536 / 12 ** 0.5) < 60

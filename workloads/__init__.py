@@ -8,6 +8,8 @@ used by both sides of the parity check without coupling them.
 """
 from .generators import (  # noqa: F401
     random_qubo,
+    random_qubo_ctr,
+    random_qubo_ctr_rows,
     maxcut_graph,
     maxcut_qubo,
     tsp_instance,

@@ -65,6 +65,84 @@ def random_qubo(n: int, seed: int = 1) -> np.ndarray:
     return W
 
 
+_TAG_RQBC = 0x52514243  # 'RQBC': counter-based random QUBO (random_qubo_ctr)
+
+
+def _philox4x32_10(c0, c1, c2, c3, k0: int, k1: int):
+    """Philox4x32-10 (Salmon et al., SC'11) over numpy uint32 arrays of
+    counters; an input generator only (the method's own draws are elsewhere)."""
+    c0, c1, c2, c3 = (np.asarray(v, dtype=np.uint32) for v in (c0, c1, c2, c3))
+    c0, c1, c2, c3 = np.broadcast_arrays(c0, c1, c2, c3)
+    k0, k1 = np.uint32(k0 & 0xFFFFFFFF), np.uint32(k1 & 0xFFFFFFFF)
+    M0, M1 = np.uint64(0xD2511F53), np.uint64(0xCD9E8D57)
+    for _ in range(10):
+        p0 = c0.astype(np.uint64) * M0
+        p1 = c2.astype(np.uint64) * M1
+        c0, c1, c2, c3 = ((p1 >> np.uint64(32)).astype(np.uint32) ^ c1 ^ k0, p1.astype(np.uint32),
+                          (p0 >> np.uint64(32)).astype(np.uint32) ^ c3 ^ k1, p0.astype(np.uint32))
+        k0 = np.uint32((int(k0) + 0x9E3779B9) & 0xFFFFFFFF)
+        k1 = np.uint32((int(k1) + 0xBB67AE85) & 0xFFFFFFFF)
+    return c0, c1, c2, c3
+
+
+def random_qubo_ctr_rows(n: int, seed: int, r0: int, r1: int) -> np.ndarray:
+    """Rows [r0, r1) of random_qubo_ctr(n, seed), without building the rest."""
+    n = int(n)
+    out = np.empty((r1 - r0, n), dtype=np.int16)
+    groups = (n + 7) // 8
+    k0, k1 = int(seed) & 0xFFFFFFFF, (int(seed) >> 32) & 0xFFFFFFFF
+    for a in range(r0, r1, 256):
+        b = min(r1, a + 256)
+        rows = np.arange(a, b, dtype=np.uint32)[:, None]
+        # upper part of row i (j >= i): the row's own stream
+        o = _philox4x32_10(rows, np.arange(groups, dtype=np.uint32)[None, :], _TAG_RQBC, 0, k0, k1)
+        up = np.stack(o, axis=-1).astype("<u4").view("<i2").reshape(b - a, groups * 8)[:, :n]
+        # lower part (j < i): W_ij = W_ji = half (i & 1) of word ((i >> 1) & 3) of the stream of row j
+        cols = np.arange(n, dtype=np.uint32)[None, :]
+        ol = _philox4x32_10(cols, (rows >> np.uint32(3)), _TAG_RQBC, 0, k0, k1)
+        words = np.stack(ol, axis=-1)                                        # [rows, n, 4]
+        sel = ((np.arange(a, b) >> 1) & 3)[:, None, None]
+        w = np.take_along_axis(words, np.broadcast_to(sel, (b - a, n, 1)), axis=2)[..., 0]
+        half = (w >> ((np.arange(a, b, dtype=np.uint32) & 1) * 16)[:, None]).astype(np.uint16).view(np.int16)
+        jj = np.arange(n)[None, :]
+        ii = np.arange(a, b)[:, None]
+        out[a - r0:b - r0] = np.where(jj >= ii, up, half)
+    return out
+
+
+def random_qubo_ctr(n: int, seed: int = 1) -> np.ndarray:
+    """Synthetic random QUBO by a counter-based rule that the
+    library also runs on the device (abs_random_qubo_dev, include/abs.h):
+    W symmetric, upper triangle (i <= j)
+        W_ij = int16 half (j & 1) of word ((j >> 1) & 3) of
+               Philox4x32-10(key = (lo32 seed, hi32 seed), counter = (i, j >> 3, 'RQBC', 0)),
+    i.i.d. uniform over all int16.  This host copy feeds the oracle; the GPU
+    side generates its replica in HBM, so a multi-GPU run stages no 2 GiB
+    host copy per rank."""
+    n = int(n)
+    if n < 1:
+        raise ValueError("n must be >= 1")
+    W = np.empty((n, n), dtype=np.int16)
+    groups = (n + 7) // 8
+    k0, k1 = int(seed) & 0xFFFFFFFF, (int(seed) >> 32) & 0xFFFFFFFF
+    B = 512
+    for r0 in range(0, n, B):
+        r1 = min(n, r0 + B)
+        g0 = r0 >> 3
+        rows = np.arange(r0, r1, dtype=np.uint32)[:, None]
+        o = _philox4x32_10(rows, np.arange(g0, groups, dtype=np.uint32)[None, :], _TAG_RQBC, 0, k0, k1)
+        U = np.stack(o, axis=-1).astype("<u4").view("<i2").reshape(r1 - r0, (groups - g0) * 8)[:, :n - 8 * g0]
+        # U[r, q] = value (r0 + r, 8 g0 + q) of the upper rule; keep j >= i
+        c0 = r0 - 8 * g0                       # column of j = r0 inside U
+        D = U[:, c0:c0 + (r1 - r0)]              # diagonal block
+        W[r0:r1, r0:r1] = np.triu(D) + np.triu(D, 1).T
+        if r1 < n:
+            R = U[:, c0 + (r1 - r0):]
+            W[r0:r1, r1:] = R
+            W[r1:, r0:r1] = R.T
+    return W
+
+
 def maxcut_graph(n: int, m_edges: int, seed: int = 1, weights: str = "pm1"):
     """G(n, m) random graph: m distinct undirected edges drawn uniformly from
     the n(n-1)/2 pairs. weights: 'pm1' (+1/-1 equiprobable, G-set G27-like)
