@@ -13,8 +13,8 @@ ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 LIB = os.path.join(HERE, "libabs.so")
 TIMING_LIB = os.path.join(HERE, "libabs_timing.so")  # diagnostics variant (-DABS_TIMING)
-SOURCES = ["abs_round.cu", "abs_setup.cu", "abs_init_mma.cu", "abs_host.cpp"]
-HEADERS = ["abs_internal.h", "philox.hpp", "ptx.cuh"]
+SOURCES = ["abs_round.cu", "abs_round_warp.cu", "abs_setup.cu", "abs_init_mma.cu", "abs_host.cpp"]
+HEADERS = ["abs_internal.h", "abs_round_common.cuh", "philox.hpp", "ptx.cuh"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 

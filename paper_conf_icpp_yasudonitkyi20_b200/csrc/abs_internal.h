@@ -123,6 +123,10 @@ int launch_wsplit(const Instance &I, int8_t *hi, uint8_t *lo, cudaStream_t st);
 int launch_init_mma(const Instance &I, const int8_t *hi, const uint8_t *lo, const uint8_t *X, int32_t row_bytes,
                     int32_t count, uint8_t *A, int64_t *E, int32_t *delta, cudaStream_t st);
 size_t round_smem_bytes(int32_t nt, int32_t bpt);
+// one-warp searches (nt == 32, n <= 2048): abs_round_warp.cu
+size_t round_warp_smem_bytes(int32_t n_pad);
+int round_warp_occupancy(int32_t bpt, int *per_sm);
+int launch_round_warp(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q, int *grid_out);
 // CTAs of the round kernel for layout (nt, bpt) resident per SM (cudaError_t).
 int round_occupancy(int32_t nt, int32_t bpt, int *per_sm);
 

@@ -33,8 +33,7 @@
 #include <climits>
 #include <cstdint>
 
-#include "abs_internal.h"
-#include "ptx.cuh"
+#include "abs_round_common.cuh"
 
 namespace absb {
 namespace {
@@ -47,105 +46,6 @@ constexpr int kWinMax = 256;
 #endif
 constexpr int kRowChunks = ABS_ROW_CHUNKS;  // bulk copies (and mbarriers) per W row: 1 or 2  // largest l served by the prefetch path (ladder max, reading C7)
 
-// Diagnostics build (-DABS_TIMING): per-warp cycle accounting of the flip loop.
-#ifdef ABS_TIMING
-#define ABS_T(x) x
-#else
-#define ABS_T(x)
-#endif
-
-template <int kP>
-struct MaskOf;
-template <>
-struct MaskOf<32> {
-    using T = uint32_t;
-};
-template <>
-struct MaskOf<64> {
-    using T = uint64_t;
-};
-
-constexpr uint32_t kTagSA = 0x5341504Cu;  // 'SAPL'
-// SA proposals evaluated per barrier (at most; the batch adapts, sa_next), <= 32 (one lane
-// per proposal).  Multi-warp searches (n > 2048) pay a CTA barrier per batch: 32 measured
-// +9.5% at n = 32k and +1.5% at n = 10,000 over 8.  One-warp searches keep 8: their CTAs
-// are small and many per SM, so the shared-memory bytes count (16 measured -1.5% at n = 1k).
-#ifndef ABS_SA_BATCH_ONE
-#define ABS_SA_BATCH_ONE 8
-#endif
-#ifndef ABS_SA_BATCH_MULTI
-#define ABS_SA_BATCH_MULTI 32
-#endif
-constexpr int kSaBatchOne = ABS_SA_BATCH_ONE, kSaBatchMulti = ABS_SA_BATCH_MULTI;
-static_assert(kSaBatchOne >= 1 && kSaBatchOne <= 32 && kSaBatchMulti >= 1 && kSaBatchMulti <= 32,
-              "one lane per proposal");
-
-// Philox4x32-10 (Salmon et al., SC'11), the library's device copy (the oracle
-// has its own; both are pinned by the Random123 known-answer vectors).
-__device__ __forceinline__ void philox4x32_10(uint32_t c0, uint32_t c1, uint32_t c2, uint32_t c3, uint32_t k0,
-                                              uint32_t k1, uint32_t (&o)[4])
-{
-#pragma unroll
-    for (int r = 0; r < 10; ++r) {
-        const uint32_t hi0 = __umulhi(0xD2511F53u, c0), lo0 = 0xD2511F53u * c0;
-        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c2), lo1 = 0xCD9E8D57u * c2;
-        c0 = hi1 ^ c1 ^ k0;
-        c1 = lo1;
-        c2 = hi0 ^ c3 ^ k1;
-        c3 = lo0;
-        k0 += 0x9E3779B9u;
-        k1 += 0xBB67AE85u;
-    }
-    o[0] = c0;
-    o[1] = c1;
-    o[2] = c2;
-    o[3] = c3;
-}
-
-// SA acceptance (Eq.(7), reading E2): an uphill move dE > 0 is
-// accepted with p = exp(-dE/(k_B t)), k_B t = tau / ln 2, i.e. p = 2^(-dE/tau);
-// the decision is u < P for a uniform uint32 u and the Q32 integer
-// P = floor(2^32 p), computed exactly in integers:
-//   2^(-dE/tau) = 2^(-q) e^(-x),  q = dE div tau,  x = ln2 (dE mod tau) / tau,
-//   e^(-x) by its Taylor series in Q63 (terms vanish by k = 19 since x < ln 2).
-constexpr uint64_t kLn2Q64 = 0xB17217F7D1CF79ABull;  // floor(ln 2 * 2^64)
-
-__device__ __noinline__ uint64_t sa_threshold_exact(int dE, int tau)
-{
-    const uint32_t ut = (uint32_t)tau;
-    const uint32_t q = (uint32_t)dE / ut;
-    const uint32_t r = (uint32_t)dE - q * ut;
-    if (q > 32) return 0;
-    // F = floor(r 2^64 / tau), Q64, by two 64/32-bit long-division steps (r < tau < 2^31)
-    const uint64_t n1 = (uint64_t)r << 32;
-    const uint64_t h = n1 / ut;
-    const uint64_t n2 = (n1 - h * ut) << 32;
-    const uint64_t F = (h << 32) | (n2 / ut);
-    const uint64_t x = __umul64hi(F, kLn2Q64);  // ln2 r / tau, Q64
-    uint64_t term = 1ull << 63, y = 1ull << 63;  // Q63
-#pragma unroll
-    for (int k = 1; k <= 20; ++k) {
-        term = __umul64hi(term, x) / (uint64_t)k;  // x^k / k!
-        y = (k & 1) ? y - term : y + term;
-    }
-    return y >> (31 + q);  // 2^32 2^(-q) y / 2^63
-}
-
-// u < P(dE, tau), deciding most draws without P: the chord C of 2^(-x) between
-// the integer exponents q and q+1 lies above the convex 2^(-x) and at most 6.2%
-// above it, so P <= C and P > 15 C / 16 - 1 (reading E2); only a
-// draw inside that band computes P.
-__device__ __forceinline__ bool sa_accept(int dE, int tau, uint32_t u)
-{
-    if (dE <= 0) return true;
-    const uint32_t q = (uint32_t)dE / (uint32_t)tau;
-    if (q > 32) return false;
-    const uint32_t r = (uint32_t)dE - q * (uint32_t)tau;
-    const long long C = (long long)(((1ull << (32 - q)) * (2ull * (uint32_t)tau - r)) / (2ull * (uint32_t)tau));
-    if ((long long)u >= C + 16) return false;
-    if ((long long)u < C - (C >> 4) - 16) return true;
-    return (uint64_t)u < sa_threshold_exact(dE, tau);
-}
 
 struct Red {
     int v;  // min Delta over all bits (neighbour tracking)
@@ -1099,157 +999,20 @@ struct Round {
     }
 };
 
-template <int kP, int kMaxT, int kNT, bool kSA>
-__global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (kMaxT == 128 ? 6 : 1)) round_kernel(const RoundArgs A)
-{
-    extern __shared__ __align__(128) unsigned char smem[];
-    const int sid = blockIdx.x;
-    const size_t bpv = (size_t)A.n_pad / 8;
-    int fbase = 0;
-    Round<kP, kMaxT, kNT, kSA>::init_barriers(smem);
-    uint8_t *const B0 = A.B + sid * bpv;
-    int64_t *const EB0 = A.EB + sid;
-    Round<kP, kMaxT, kNT, kSA>::run(
-        A, smem, sid, A.T + sid * bpv,
-        [=](uint8_t *&Bp, int64_t *&EBp) {
-            Bp = B0;
-            EBp = EB0;
-        },
-        fbase);
-}
-
-// ---------------------------------------------------------------- asynchronous mode
-__device__ __forceinline__ uint32_t ld_acquire_sys(const uint32_t *p)
-{
-    uint32_t v;
-    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_release_sys(uint32_t *p, uint32_t v)
-{
-    asm volatile("st.release.sys.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-__device__ __forceinline__ int ld_acquire_gpu(const int *p)
-{
-    int v;
-    asm volatile("ld.acquire.gpu.global.s32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
-    return v;
-}
-__device__ __forceinline__ void st_release_gpu(int *p, int v)
-{
-    asm volatile("st.release.gpu.global.s32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
-}
-
-// The paper's device loop (Steps 2-5 repeated) as a persistent
-// kernel.  When every search fits on the GPU (S <= resident CTAs) CTA b owns
-// search b and draws round tickets from a shared budget, so each search runs
-// at its own pace ("each CUDA block operates asynchronously");
-// otherwise CTAs take (search, round) items from a queue.  A round reads the
-// search's latest target from mapped host memory (Step 2; a stale target is
-// reused, reading C11) and publishes (B, E_B) to mapped host memory with a
-// system-scope release and appends (search, round) to an arrival ring the host
-// GA polls.
-// Host and device never synchronise directly.
-template <int kP, int kMaxT, int kNT, bool kSA>
-__global__ void __launch_bounds__(kMaxT, kMaxT == 32 ? (kP == 32 ? 32 : 16) : (kMaxT == 128 ? 6 : 1))
-    round_kernel_async(const RoundArgs A, const AsyncArgs Q)
-{
-    extern __shared__ __align__(128) unsigned char smem[];
-    // the current work item, kept in shared memory so that nothing of it stays
-    // live in registers across the flip loop
-    __shared__ long long item;
-    __shared__ int cur_s, cur_r, r_own;
-    __shared__ uint32_t tver;
-    const size_t bpv = (size_t)A.n_pad / 8;
-    constexpr bool multi = kMaxT > 32;
-    int fbase = 0;
-    Round<kP, kMaxT, kNT, kSA>::init_barriers(smem);
-    if (threadIdx.x == 0) r_own = Q.owned ? ld_acquire_gpu(Q.done + blockIdx.x) : 0;
-    for (;;) {
-        if (threadIdx.x == 0) {
-            const long long q = (long long)atomicAdd(Q.queue, 1ull);
-            item = q;
-            if (q < Q.total) {
-                const int s = Q.owned ? (int)blockIdx.x : (int)(q % A.S);
-                const int r = Q.owned ? r_own++ : Q.base + (int)(q / A.S);
-                ABS_T(const long long w0 = clock64();)
-                if (!Q.owned)
-                    while (ld_acquire_gpu(Q.done + s) != r) __nanosleep(256);  // round r-1 of s finished
-                ABS_T(const long long w1 = clock64();)
-                // the result slot of round r (double-buffered) must have been consumed by the host
-                while ((int)ld_acquire_sys(Q.rack + s) < r - 1) __nanosleep(1024);
-                ABS_T(const long long w2 = clock64();)
-                tver = ld_acquire_sys(Q.tseq + s);  // latest published target version
-                cur_s = s;
-                cur_r = r;
-                ABS_T(if (A.timing) {
-                    unsigned long long *tm = (unsigned long long *)&A.timing[((size_t)s * 32) * 24];
-                    atomicAdd(tm + 16, (unsigned long long)(w1 - w0));
-                    atomicAdd(tm + 17, (unsigned long long)(w2 - w1));
-                    atomicAdd(tm + 18, (unsigned long long)(clock64() - w2));
-                    atomicAdd(tm + 20, 1ull);
-                })
-            }
-        }
-        if (multi) __syncthreads();
-        else __syncwarp();
-        if (item >= Q.total) break;
-        Round<kP, kMaxT, kNT, kSA>::run(
-            A, smem, cur_s, Q.Tmap + ((size_t)cur_s * 2 + (tver & 1)) * bpv,
-            [&](uint8_t *&Bp, int64_t *&EBp) {
-                const int s = cur_s, r = cur_r;
-                Bp = Q.Rb + ((size_t)s * 2 + (r & 1)) * bpv;
-                EBp = Q.Reb + (size_t)s * 2 + (r & 1);
-            },
-            fbase);
-        if (threadIdx.x == 0) Q.rtver[(size_t)cur_s * 2 + (cur_r & 1)] = tver;
-        __threadfence_system();  // B, E_B and the target version reach host memory ...
-        if (multi) __syncthreads();
-        else __syncwarp();
-        if (threadIdx.x == 0) {
-            ABS_T(const long long p0 = clock64();)
-            const int s = cur_s, r = cur_r;
-            // arrival ring: the host GA drains results in this order.  The
-            // index comes from a DEVICE counter: a system-scope atomic on host memory
-            // serialises every CTA over PCIe (~1M results/s for the whole GPU)
-            const uint32_t idx = atomicAdd(Q.rcount, 1u);
-            Q.ring[2 * (idx & Q.ring_mask)] = (uint32_t)s;
-            Q.ring[2 * (idx & Q.ring_mask) + 1] = (uint32_t)r;
-            st_release_sys(Q.ringseq + (idx & Q.ring_mask), idx + 1u);  // ... before the ring entry
-            st_release_gpu(Q.done + s, r + 1);
-            ABS_T(if (A.timing) atomicAdd((unsigned long long *)&A.timing[((size_t)s * 32) * 24 + 19],
-                                          (unsigned long long)(clock64() - p0));)
-        }
-    }
-}
+// resident CTAs per SM the register budget is sized for (launch bounds)
+constexpr int min_blocks(int p, int max_t) { return max_t == 32 ? (p == 32 ? 32 : 16) : (max_t == 128 ? 6 : 1); }
 
 template <int kP, int kMaxT, int kNT, bool kSA>
 int launch_policy(const RoundArgs &a, cudaStream_t st, size_t smem, const AsyncArgs *q, int *grid_out)
 {
-    if (!q) {
-        auto k = round_kernel<kP, kMaxT, kNT, kSA>;
-        cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-        k<<<a.S, a.nt, smem, st>>>(a);
-        return (int)cudaGetLastError();
-    }
-    auto k = round_kernel_async<kP, kMaxT, kNT, kSA>;
-    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    int per_sm = 0, dev = 0, sms = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, a.nt, smem);
-    const int grid = (int)std::min<long long>((long long)a.S, (long long)std::max(1, per_sm) * sms);
-    if (grid_out) *grid_out = grid;
-    AsyncArgs q2 = *q;
-    q2.owned = grid >= a.S ? 1 : 0;
-    k<<<grid, a.nt, smem, st>>>(a, q2);
-    return (int)cudaGetLastError();
+    return launch_kernel<Round<kP, kMaxT, kNT, kSA>, kMaxT, min_blocks(kP, kMaxT)>(a, st, smem, q, grid_out);
 }
 
 }  // namespace
 
 size_t round_smem_bytes(int32_t nt, int32_t bpt)
 {
+    if (nt == 32) return round_warp_smem_bytes(32 * bpt);  // one-warp searches: abs_round_warp.cu
     const bool multi = nt > 32;
     const size_t msz = bpt == 64 ? 8 : 4;
     size_t s = (multi ? sizeof(RoundSmemT<kSaBatchMulti>) + sizeof(WindowSmem) : sizeof(RoundSmemT<kSaBatchOne>)) +
@@ -1268,19 +1031,16 @@ int launch_variant(const RoundArgs &a, cudaStream_t st, size_t smem, const Async
 template <int kP, int kMaxT, int kNT>
 int occupancy_variant(int nt, size_t smem, int *per_sm)
 {
-    auto k = round_kernel<kP, kMaxT, kNT, false>;
-    cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    return (int)cudaOccupancyMaxActiveBlocksPerMultiprocessor(per_sm, k, nt, smem);
+    return occupancy_of<Round<kP, kMaxT, kNT, false>, kMaxT, min_blocks(kP, kMaxT)>(nt, smem, per_sm);
 }
 
 int round_occupancy(int32_t nt, int32_t bpt, int *per_sm)
 {
+    if (nt == 32) return round_warp_occupancy(bpt, per_sm);  // one-warp searches: abs_round_warp.cu
     const size_t smem = round_smem_bytes(nt, bpt);
     if (bpt == 32) {
-        if (nt == 32) return occupancy_variant<32, 32, 32>(nt, smem, per_sm);
         return occupancy_variant<32, 128, 0>(nt, smem, per_sm);
     }
-    if (nt == 32) return occupancy_variant<64, 32, 32>(nt, smem, per_sm);  // n_pad = 2048
     if (nt == 512) return occupancy_variant<64, 512, 512>(nt, smem, per_sm);
     if (nt == 160) return occupancy_variant<64, 512, 160>(nt, smem, per_sm);  // n_pad = 10240 (TSP, 100 cities)
     return occupancy_variant<64, 512, 0>(nt, smem, per_sm);
@@ -1288,12 +1048,11 @@ int round_occupancy(int32_t nt, int32_t bpt, int *per_sm)
 
 int launch_round(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q, int *grid_out)
 {
+    if (a.nt == 32) return launch_round_warp(a, st, q, grid_out);  // one-warp searches: abs_round_warp.cu
     const size_t smem = round_smem_bytes(a.nt, a.bpt);
     if (a.bpt == 32) {
-        if (a.nt == 32) return launch_variant<32, 32, 32>(a, st, smem, q, grid_out);
         return launch_variant<32, 128, 0>(a, st, smem, q, grid_out);  // nt = 96
     }
-    if (a.nt == 32) return launch_variant<64, 32, 32>(a, st, smem, q, grid_out);  // n_pad = 2048
     if (a.nt == 512) return launch_variant<64, 512, 512>(a, st, smem, q, grid_out);  // n_pad = 32768
     if (a.nt == 160) return launch_variant<64, 512, 160>(a, st, smem, q, grid_out);  // n_pad = 10240 (TSP, 100 cities)
     return launch_variant<64, 512, 0>(a, st, smem, q, grid_out);

@@ -25,6 +25,12 @@ for line in out.splitlines():
     if m:
         rows[cur]["reg"] = int(m.group(1))
 def short(name):
+    m = re.search(r"(round_kernel(?:_async)?)I.*?5RoundILi(\d+)ELi(\d+)ELi(\d+)ELb(\d)", name)
+    if m:
+        return "%s<%s,%s,%s,%s>" % (m.group(1), m.group(2), m.group(3), m.group(4), "SA" if m.group(5) == "1" else "win")
+    m = re.search(r"(round_kernel(?:_async)?)I.*?9WarpRoundILi(\d+)ELb(\d)", name)
+    if m:
+        return "%s<warp %s,%s>" % (m.group(1), m.group(2), "SA" if m.group(3) == "1" else "win")
     m = re.search(r"(round_kernel(?:_async)?)ILi(\d+)ELi(\d+)ELi(\d+)ELb(\d)", name)
     if m:
         return "%s<%s,%s,%s,%s>" % (m.group(1), m.group(2), m.group(3), m.group(4), "SA" if m.group(5) == "1" else "win")
