@@ -570,7 +570,7 @@ def main():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sub", action="store_true", help="skip the configs 2-4 sub-results")
-    ap.add_argument("--sub-seconds", type=float, default=2.5)
+    ap.add_argument("--sub-seconds", type=float, default=3.0)
     ap.add_argument("--async-seconds", type=float, default=10.0)
     ap.add_argument("--cpu-seconds", type=float, default=15.0)
     ap.add_argument("--ref-step-seconds", type=float, default=8.0)
