@@ -507,6 +507,144 @@ struct Round {
         return acc;
     }
 
+    // Window-first selection of the next local flip by the controller warp (the last
+    // warp): applies row k_f (buffer b) to the published Delta(X_f) of window
+    // W_{f+1} = {(a + l + r) mod n : r < l}, takes the lowest-index argmin
+    // (reading C5), issues the TMA of row k_{f+1} into buffer b ^ 1 and leaves
+    // (k_{f+1}, Delta, x, 1) in sel[b].
+    static __device__ __forceinline__ void window_first(const RoundArgs &A, RoundSmem *sm, const WindowSmem *win,
+                                                        unsigned char *rowbuf, size_t rowb, int b, uint32_t par,
+                                                        int a, int l, int n, int xk, int lane, int warp, int nt,
+                                                        long long tc0)
+    {
+        (void)warp;
+        (void)tc0;
+        const unsigned char *row = rowbuf + rowb * b;
+        int a1 = a + l;
+        if (a1 >= n) a1 -= n;
+        {
+            // wait for the half rows of row k_f that hold the window's bits
+            const int end = a1 + l - 1;
+            const int h0 = group_of(a1, nt) / (G / 2);
+            const int h1 = (end >= n) ? 1 : group_of(end, nt) / (G / 2);
+            if (kRowChunks == 1) {
+                mbar_wait(&sm->bar[b][0], par);
+            } else {
+                if (end >= n || h0 == 0) mbar_wait(&sm->bar[b][0], par);
+                if (h1 == 1) mbar_wait(&sm->bar[b][1], par);
+            }
+        }
+        ABS_T(const long long ts1 = clock64();)
+        const int *wd = win->d[b];
+        const uint8_t *wx = win->x[b];
+        const short *rw = reinterpret_cast<const short *>(row);
+        // key = (Delta_i(X_{f+1}) << 32) | (2i + x_i): its minimum is the
+        // lowest-index argmin (reading C5) and carries x_i along
+        long long best = LLONG_MAX;
+        // l <= kWinMax = 8 * 32: a lane's loads are issued in batches of four;
+        // batches wholly beyond l are skipped (warp-uniform)
+#pragma unroll
+        for (int h = 0; h < kWinMax / 128; ++h) {
+            if (h > 0 && 128 * h >= l) break;
+            int dd[4], ww[4], xx[4], ii[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int r = lane + 32 * (4 * h + q);
+                int i = a1 + r;
+                if (i >= n) i -= n;
+                ii[q] = i;
+                dd[q] = 0;
+                xx[q] = 0;
+                ww[q] = 0;
+                if (r < l) {
+                    dd[q] = wd[r];
+                    xx[q] = wx[r];
+                    ww[q] = rw[i];
+                }
+            }
+            // k_f is not in this window (windows are disjoint: l <= kWinMax <= n/8 here),
+            // so every entry moves by Eq.(16); the four keys are reduced as a tree
+            long long kq[4];
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+                const int d = dd[q] + ww[q] * (2 - 4 * (xx[q] ^ xk));  // Eq.(16)
+                kq[q] = (lane + 32 * (4 * h + q) < l)
+                            ? (long long)(((unsigned long long)(unsigned)d << 32) | (unsigned)(2 * ii[q] + xx[q]))
+                            : LLONG_MAX;
+            }
+            best = min(best, min(min(kq[0], kq[1]), min(kq[2], kq[3])));
+        }
+        const int bv = (int)(best >> 32);
+        ABS_T(const long long ts2 = clock64();)
+        const int mv = __reduce_min_sync(kFull, bv);
+        const int mi = __reduce_min_sync(kFull, bv == mv ? (int)(unsigned)best : INT_MAX);
+        ABS_T(const long long ts3 = clock64();)
+        // the warp is converged here: one elected lane issues (no per-lane loop
+        // around the bulk copy's uniform operands)
+        if (elect_one()) issue_row(A, mi >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
+        if (lane == 0) sm->sel[b] = make_int4(mi >> 1, mv, mi & 1, 1);
+        ABS_T(if (lane == 0) {
+            const long long ts4 = clock64();
+            sm->tacc[warp][16] += ts1 - tc0;  // wait for row k_f's window half
+            sm->tacc[warp][17] += ts2 - ts1;  // window arithmetic
+            sm->tacc[warp][18] += ts3 - ts2;  // two warp reductions
+            sm->tacc[warp][19] += ts4 - ts3;  // TMA issue + sel
+            sm->tacc[warp][20] += 1;
+        })
+    }
+
+    // The hot loop of the window policy at n > 2048: consecutive NON-exact local flips
+    // with the window-first prefetch.  The general flip body of run() with the
+    // straight, SA and exact-tracking branches compiled out, so each warp issues
+    // little besides its row update (Eq.(16)).  Entered at the start of flip f with
+    // row k_f in flight; returns at the start of the first flip that is exact or
+    // has no local successor (left <= 1), in the state the general body expects.
+    static __device__ __forceinline__ void fast_local(const RoundArgs &A, RoundSmem *sm, WindowSmem *win,
+                                                      unsigned char *rowbuf, size_t rowb, int (&g)[kP], M &xm,
+                                                      int &a, int l, int n, int t, int nt, int lane, int warp, int nw,
+                                                      int ctl, int &left, int &k, int &dk, int &xk, bool &exact,
+                                                      int &f, int fbase)
+    {
+        const long long wmax2 = 2 * (long long)A.wmax;
+        while (!exact && left > 1) {
+            const int b = (fbase + f) & 1;
+            const uint32_t par = (uint32_t)((fbase + f) >> 1) & 1u;
+            if (warp == nw - 1) window_first(A, sm, win, rowbuf, rowb, b, par, a, l, n, xk, lane, warp, nt, 0);
+            const int c = xk ? -2 : 2;  // 2 phi(x_k), pre-flip bit (Eq.(16))
+            {
+                const int j = group_of(k, nt);
+                if (t == (k >> 3) - nt * j) xm ^= (M)1 << (8 * j + (k & 7));  // x_k <- 1 - x_k
+            }
+            int vmin, vj, cmin, cj;
+            process_row<kUpdate>(g, xm, 0, reinterpret_cast<const uint4 *>(rowbuf + rowb * b), sm->bar[b], par, c, t,
+                                 nt, vmin, vj, cmin, cj);
+            a += l;  // offset <- (a + l) mod n
+            if (a >= n) a -= n;
+            int a2 = a + l;
+            if (a2 >= n) a2 -= n;
+            publish_window(g, xm, a2, l, n, t, nt, win->d[b ^ 1], win->x[b ^ 1]);
+            if (t == ctl) {  // E(X') = E(X) + d_k, the bound LB, lazy tracking of flip f+1
+                sm->hash = (sm->hash ^ (uint64_t)(uint32_t)k) * kFnvPrime;
+                sm->nflip += 1;
+                const long long E1 = sm->E + dk;
+                const long long LB1 = min(sm->LB - wmax2, -(long long)dk);
+                sm->E = E1;
+                sm->LB = LB1;
+                const int dk1 = sm->sel[b].y;
+                const long long LB2 = min(LB1 - wmax2, -(long long)dk1);
+                sm->sel[b].w = (E1 + dk1 + min(LB2, 0LL) < sm->EB) ? 1 : 0;
+            }
+            __syncthreads();  // row buffer b free; sel[b] and the window published
+            --left;
+            const int4 sv = sm->sel[b];
+            k = sv.x;
+            dk = sv.y;
+            xk = sv.z;
+            exact = sv.w != 0;
+            ++f;
+        }
+    }
+
     static __device__ __forceinline__ void init_barriers(unsigned char *smem)
     {
         RoundSmem *sm = reinterpret_cast<RoundSmem *>(smem);
@@ -618,85 +756,21 @@ struct Round {
         int f = 0;
         ABS_T(if (lane == 0) for (int q = 0; q < 24; ++q) sm->tacc[warp][q] = 0;)
         for (; have; ++f) {
+#ifndef ABS_TIMING
+            if constexpr (kMulti && !kSA) {
+                if (pre && !straight)
+                    fast_local(A, sm, win, rowbuf, rowb, g, xm, a, l, n, t, nt, lane, warp, nw, ctl, left, k, dk, xk,
+                               exact, f, fbase);
+            }
+#endif
             const int b = (fbase + f) & 1;
             const uint32_t par = (uint32_t)((fbase + f) >> 1) & 1u;
             unsigned char *row = rowbuf + rowb * b;
             ABS_T(long long tc0 = clock64(); const int to = straight ? 8 : 0;)
 
             // ---- window-first selection of the next flip (the last warp, the controller), prefetch its row
-            if (pre && !straight && left > 1 && warp == nw - 1) {
-                int a1 = a + l;
-                if (a1 >= n) a1 -= n;
-                {
-                    // wait for the half rows of row k_f that hold the window's bits
-                    const int end = a1 + l - 1;
-                    const int h0 = group_of(a1, nt) / (G / 2);
-                    const int h1 = (end >= n) ? 1 : group_of(end, nt) / (G / 2);
-                    if (kRowChunks == 1) {
-                        mbar_wait(&sm->bar[b][0], par);
-                    } else {
-                        if (end >= n || h0 == 0) mbar_wait(&sm->bar[b][0], par);
-                        if (h1 == 1) mbar_wait(&sm->bar[b][1], par);
-                    }
-                }
-                ABS_T(const long long ts1 = clock64();)
-                const int *wd = win->d[b];
-                const uint8_t *wx = win->x[b];
-                const short *rw = reinterpret_cast<const short *>(row);
-                // key = (Delta_i(X_{f+1}) << 32) | (2i + x_i): its minimum is the
-                // lowest-index argmin (reading C5) and carries x_i along
-                long long best = LLONG_MAX;
-                // l <= kWinMax = 8 * 32: a lane's loads are issued in batches of four;
-                // batches wholly beyond l are skipped (warp-uniform)
-#pragma unroll
-                for (int h = 0; h < kWinMax / 128; ++h) {
-                    if (h > 0 && 128 * h >= l) break;
-                    int dd[4], ww[4], xx[4], ii[4];
-#pragma unroll
-                    for (int q = 0; q < 4; ++q) {
-                        const int r = lane + 32 * (4 * h + q);
-                        int i = a1 + r;
-                        if (i >= n) i -= n;
-                        ii[q] = i;
-                        dd[q] = 0;
-                        xx[q] = 0;
-                        ww[q] = 0;
-                        if (r < l) {
-                            dd[q] = wd[r];
-                            xx[q] = wx[r];
-                            ww[q] = rw[i];
-                        }
-                    }
-                    // k_f is not in this window (windows are disjoint: l <= kWinMax <= n/8 here),
-                    // so every entry moves by Eq.(16); the four keys are reduced as a tree
-                    long long kq[4];
-#pragma unroll
-                    for (int q = 0; q < 4; ++q) {
-                        const int d = dd[q] + ww[q] * (2 - 4 * (xx[q] ^ xk));  // Eq.(16)
-                        kq[q] = (lane + 32 * (4 * h + q) < l)
-                                    ? (long long)(((unsigned long long)(unsigned)d << 32) | (unsigned)(2 * ii[q] + xx[q]))
-                                    : LLONG_MAX;
-                    }
-                    best = min(best, min(min(kq[0], kq[1]), min(kq[2], kq[3])));
-                }
-                const int bv = (int)(best >> 32);
-                ABS_T(const long long ts2 = clock64();)
-                const int mv = __reduce_min_sync(kFull, bv);
-                const int mi = __reduce_min_sync(kFull, bv == mv ? (int)(unsigned)best : INT_MAX);
-                ABS_T(const long long ts3 = clock64();)
-                // the warp is converged here: one elected lane issues (no per-lane loop
-                // around the bulk copy's uniform operands)
-                if (elect_one()) issue_row(A, mi >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
-                if (lane == 0) sm->sel[b] = make_int4(mi >> 1, mv, mi & 1, 1);
-                ABS_T(if (lane == 0) {
-                    const long long ts4 = clock64();
-                    sm->tacc[warp][16] += ts1 - tc0;  // wait for row k_f's window half
-                    sm->tacc[warp][17] += ts2 - ts1;  // window arithmetic
-                    sm->tacc[warp][18] += ts3 - ts2;  // two warp reductions
-                    sm->tacc[warp][19] += ts4 - ts3;  // TMA issue + sel
-                    sm->tacc[warp][20] += 1;
-                })
-            }
+            if (pre && !straight && left > 1 && warp == nw - 1)
+                window_first(A, sm, win, rowbuf, rowb, b, par, a, l, n, xk, lane, warp, nt, ABS_T(tc0) + 0);
 
             // ---- SA early decision (the SA analogue of the window-first selection): the
             // proposals left over from the batch that accepted k_f were drawn already;
