@@ -39,8 +39,8 @@ def build(force: bool = False, verbose: bool = False, timing: bool = False) -> s
         return LIB
     tmp = lib + ".tmp%d" % os.getpid()
     cmd = [nvcc(), *ARCH, *(["-DABS_TIMING"] if timing else []), "-O3", "-lineinfo", "-std=c++17", "-shared", "-Xcompiler", "-fPIC",
-           "-Xcompiler", "-fvisibility=hidden", "-I", os.path.join(ROOT, "include"), "-I", CSRC,
-           "-o", tmp] + [os.path.join(CSRC, f) for f in SOURCES] + ["-lpthread"]
+           "-Xcompiler", "-fvisibility=hidden", "-Xcompiler", "-fopenmp", "-I", os.path.join(ROOT, "include"), "-I", CSRC,
+           "-o", tmp] + [os.path.join(CSRC, f) for f in SOURCES] + ["-lpthread", "-lgomp"]
     if verbose:
         print(" ".join(cmd), file=sys.stderr)
     subprocess.check_call(cmd)

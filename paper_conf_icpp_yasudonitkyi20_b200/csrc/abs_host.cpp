@@ -129,7 +129,9 @@ static void ga_target(const Pool &P, const GaParams &ga, int64_t r, int64_t sid,
 
 // Run f(i) for i in [0, count) on up to min(16, cores) host threads; serial below
 // `grain` items.  Used for the GA targets of a lockstep step, which only READ the pool
-// (each target is a function of the pool, the round and the search id alone).
+// (each target is a function of the pool, the round and the search id alone).  An
+// OpenMP team persists between steps (spawning std::threads every step cost about as
+// much as the targets themselves at 10,000 searches).
 template <class F>
 static void parallel_for(int count, int grain, const F &f)
 {
@@ -139,15 +141,8 @@ static void parallel_for(int count, int grain, const F &f)
         for (int i = 0; i < count; ++i) f(i);
         return;
     }
-    std::vector<std::thread> th;
-    th.reserve(nth - 1);
-    auto chunk = [&](int w) {
-        const int lo = (int)((int64_t)count * w / nth), hi = (int)((int64_t)count * (w + 1) / nth);
-        for (int i = lo; i < hi; ++i) f(i);
-    };
-    for (int w = 1; w < nth; ++w) th.emplace_back(chunk, w);
-    chunk(0);
-    for (auto &x : th) x.join();
+#pragma omp parallel for num_threads(nth) schedule(static)
+    for (int i = 0; i < count; ++i) f(i);
 }
 
 }  // namespace absb
