@@ -41,10 +41,15 @@ namespace {
 constexpr uint64_t kFnvPrime = 0x100000001b3ull;
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWinMax = 256;
+// bulk copies (and mbarriers) per W row: 1, or 2 half rows (the controller starts the
+// window-first selection when the half holding the window lands).  Measured: 2 for the
+// n = 32768 variant (+1.7%), 1 elsewhere (2 cost TSP n = 10,000 8%).
+#ifndef ABS_ROW_CHUNKS_32K
+#define ABS_ROW_CHUNKS_32K 2
+#endif
 #ifndef ABS_ROW_CHUNKS
 #define ABS_ROW_CHUNKS 1
 #endif
-constexpr int kRowChunks = ABS_ROW_CHUNKS;  // bulk copies (and mbarriers) per W row: 1 or 2  // largest l served by the prefetch path (ladder max, reading C7)
 
 
 struct Red {
@@ -83,6 +88,7 @@ template <int kP, int kMaxT, int kNT, bool kSA>
 struct Round {
     static constexpr int G = kP / 8;  // byte-groups per thread
     static constexpr bool kMulti = kMaxT > 32;
+    static constexpr int kRowChunks = kNT == 512 ? ABS_ROW_CHUNKS_32K : ABS_ROW_CHUNKS;
     static constexpr int kSaBatch = kMulti ? kSaBatchMulti : kSaBatchOne;
     using RoundSmem = RoundSmemT<kSaBatch>;
     // B's neighbour bit i* from the owner of the byte-group the reduction names
