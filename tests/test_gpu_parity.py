@@ -319,7 +319,10 @@ def _replay_async(W, s, L, trace_s, l):
     return oracle.replay_search(W, l, L, T)
 
 
-@pytest.mark.parametrize("n,S,L,steps", [(300, 6, 120, 5), (1500, 4, 300, 3), (64, 6000, 40, 2)])
+@pytest.mark.parametrize("n,S,L,steps", [(300, 6, 120, 5), (1500, 4, 300, 3), (64, 6000, 40, 2),
+                                         (3000, 5, 900, 3),      # multi-warp (three warps): the hot loop
+                                         (10000, 3, 2000, 2),    # NT = 160
+                                         (32768, 2, 3000, 2)])   # NT = 512, two half-row copies
 def test_async_rounds_replay_bitexact(n, S, L, steps):
     """Async mode: timing decides which target each round gets, but given the
     targets a search actually used (trace), its trajectory is determined: the
