@@ -130,3 +130,15 @@ def test_elite_exchange_rank_order_and_padding(tmp_path):
         z = np.load(os.path.join(tmp_path, "e%d.npz" % r))
         assert z["E"].tolist() == [-100, -5, -200, -10]      # rank order, +inf padding removed
         assert z["X"][:, 0].tolist() == [1, 7, 2, 8]
+
+
+def test_bench_refuses_gpus_world_mismatch():
+    """bench.py --gpus N under a launcher with WORLD_SIZE != N must refuse to run
+    (one process per GPU), instead of silently timing a different world."""
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    env = dict(os.environ, WORLD_SIZE="3", RANK="0", LOCAL_RANK="0")
+    p = subprocess.run([sys.executable, os.path.join(root, "bench.py"), "--gpus", "2", "--steps", "1"],
+                       env=env, capture_output=True, text=True, timeout=120)
+    assert p.returncode == 2 and "WORLD_SIZE" in p.stderr

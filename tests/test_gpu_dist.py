@@ -110,3 +110,40 @@ def test_two_ranks_async_elite_exchange(tmp_path):
     W = random_qubo(500, 44)
     Xb = z[0]["X1"][0]
     assert oracle.energy(W, Xb) == best
+
+
+def _nccl_worker(rank, world, port, out_dir):
+    import paper_conf_icpp_yasudonitkyi20_b200 as pkg
+    from paper_conf_icpp_yasudonitkyi20_b200 import dist as pdist
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", init_method="tcp://127.0.0.1:%d" % port, rank=rank, world_size=world,
+                            device_id=torch.device("cuda", 0))
+    n, S, R, L = 300, 4, 2, 150
+    W = random_qubo(n, 32)
+    s = pkg.Solver(W, searches=S, external_merge=True, local_flips=L, pool_size=8, seed=10)
+    Es = []
+    for _ in range(R):
+        _, E = pdist.lockstep_step(s)   # all_gather_into_tensor over NCCL on cuda:0
+        Es.append(E)
+    PX, PE = s.pool(8)
+    ins = pdist.exchange_elites(s, 4)
+    np.savez(os.path.join(out_dir, "nccl%d.npz" % rank), E=np.array(Es), PX=PX, PE=PE, ins=ins,
+             backend=np.array([dist.get_backend()]))
+    s.close()
+    dist.destroy_process_group()
+
+
+def test_nccl_backend_single_rank(tmp_path):
+    """The NCCL path of dist.py (device tensors, all_gather_into_tensor) with a
+    one-rank communicator on cuda:0 -- NCCL refuses two ranks on one device, so
+    this is the only NCCL execution a one-GPU box allows.  The run equals the
+    one-process oracle."""
+    tmp.spawn(_nccl_worker, args=(1, _free_port(), str(tmp_path)), nprocs=1, join=True)
+    z = np.load(os.path.join(tmp_path, "nccl0.npz"))
+    assert str(z["backend"][0]) == "nccl"
+    W = random_qubo(300, 32)
+    o = oracle.run_lockstep(W, oracle.Config(n=300, searches=4, local_flips=150, pool_size=8, seed=10), 2)
+    fin = o["poolE"] != oracle.EINF
+    assert (z["E"] == o["EB"]).all()
+    assert (z["PE"] == o["poolE"][fin]).all() and (z["PX"] == o["poolX"][fin]).all()
+    assert int(z["ins"]) == 0
