@@ -86,19 +86,12 @@ struct WindowSmem {  // published Delta / x of the next window, by flip parity
 
 template <int kP, int kMaxT, int kNT, bool kSA>
 struct Round {
+    static_assert(kMaxT > 32, "searches of one warp (n <= 2048) run WarpRound (abs_round_warp.cu)");
     static constexpr int G = kP / 8;  // byte-groups per thread
-    static constexpr bool kMulti = kMaxT > 32;
     static constexpr int kRowChunks = kNT == 512 ? ABS_ROW_CHUNKS_32K : ABS_ROW_CHUNKS;
-    static constexpr int kSaBatch = kMulti ? kSaBatchMulti : kSaBatchOne;
+    static constexpr int kSaBatch = kSaBatchMulti;
     using RoundSmem = RoundSmemT<kSaBatch>;
-    // B's neighbour bit i* from the owner of the byte-group the reduction names
-    // (no second reduction); else every thread scans its slots and a second
-    // reduction picks the lowest index
-    // (multi-warp kernels: measured slower at n = 32k, code generation of the flip loop)
-    static constexpr bool kOwnerB = !kMulti;
-    // SA early decision (run()): off for one warp x 64 bits (n_pad = 2048), where it
-    // measured slower (MaxCut's high acceptance leaves few leftover proposals)
-    static constexpr bool kSaEarly = kSA && (kMulti || kP == 32);
+    static constexpr bool kSaEarly = kSA;  // SA early decision (run())
     using M = typename MaskOf<kP>::T;
 
     // ---------------------------------------------------------------- small helpers
@@ -169,52 +162,15 @@ struct Round {
         ci2 = cs < 0 ? INT_MAX : 2 * slot_index(t, nt, cs) + (int)bit(xm, cs);
     }
 
-    // candidates() over the window {(a + r) mod n : r < l} (Fig. 2),
-    // visiting only the byte-groups j the window touches (block-uniform) and
-    // skipping a group in warps that own none of its window bits.
-    static __device__ __forceinline__ void candidates_window(const int (&g)[kP], M xm, int a, int l, int n, int t,
-                                                             int nt, int &cv, int &ci2)
-    {
-        const int end = a + l;  // exclusive; > n when the window wraps (reading C6)
-        const int hi1 = min(end, n);
-        const int hi2 = end - n;
-        const int j0 = group_of(a, nt), j1 = group_of(hi1 - 1, nt);
-        const int jw = hi2 > 0 ? group_of(hi2 - 1, nt) : -1;
-        cv = INT_MAX;
-        int cs = -1;
-#pragma unroll
-        for (int j = 0; j < G; ++j) {
-            if ((j < j0 || j > j1) && j > jw) continue;
-            const int base = 8 * (t + nt * j);
-            uint32_t m = 0;
-            if (base + 8 > a && base < hi1) m |= range8(base, a, hi1);
-            if (base < hi2) m |= range8(base, 0, hi2);
-            if (!__any_sync(kFull, m != 0)) continue;
-#pragma unroll
-            for (int e = 0; e < 8; ++e) {
-                const int d = readout(g[8 * j + e], xm, 8 * j + e);
-                if (((m >> e) & 1u) && d < cv) {
-                    cv = d;
-                    cs = 8 * j + e;
-                }
-            }
-        }
-        ci2 = cs < 0 ? INT_MAX : 2 * slot_index(t, nt, cs) + (int)bit(xm, cs);
-    }
-
-    // Window argmin: one warp scans only the window's byte-groups; the
-    // multi-warp kernels keep the mask form (measured faster there, n = 32k).
+    // Window argmin over {(a + r) mod n : r < l} (Fig. 2) in the mask form
+    // (measured faster than a byte-group scan at n = 32k).
     static __device__ __forceinline__ void window_candidates(const int (&g)[kP], M xm, int a, int l, int n, int t,
                                                              int nt, int &cv, int &ci2)
     {
-        if constexpr (kMulti) {
-            const M cm = window_mask(a, l, n, t, nt);
-            cv = INT_MAX;
-            ci2 = INT_MAX;
-            if (__any_sync(kFull, cm != 0)) candidates(g, xm, cm, t, nt, cv, ci2);
-        } else {
-            candidates_window(g, xm, a, l, n, t, nt, cv, ci2);
-        }
+        const M cm = window_mask(a, l, n, t, nt);
+        cv = INT_MAX;
+        ci2 = INT_MAX;
+        if (__any_sync(kFull, cm != 0)) candidates(g, xm, cm, t, nt, cv, ci2);
     }
 
     // 2*index + x of the lowest slot in `cm` whose Delta equals v (INT_MAX if none).
@@ -231,23 +187,12 @@ struct Round {
 
     // CTA-wide min reduction (three keys); all threads get the result.  Lowest
     // index wins ties (reading C5).  Alternating slots -> one barrier per call.
-    // kOwnerB: vb = lowest byte-group holding a bit whose Delta is the minimum v
-    // (rvb: this thread's first such group, INT_MAX if none).
-    static __device__ __forceinline__ Red block_reduce(Red r, Red (*sred)[32], int &rb, int lane, int warp, int nw,
-                                                       int rvb = INT_MAX, int *vb = nullptr)
+    static __device__ __forceinline__ Red block_reduce(Red r, Red (*sred)[32], int &rb, int lane, int warp, int nw)
     {
         Red w;
         w.v = __reduce_min_sync(kFull, r.v);
         w.c = __reduce_min_sync(kFull, r.c);
         w.i = __reduce_min_sync(kFull, r.c == w.c ? r.i : INT_MAX);
-        if constexpr (kOwnerB) {
-            static_assert(!kMulti, "byte-group of the minimum: one-warp searches only");
-            if (vb) *vb = __reduce_min_sync(kFull, r.v == w.v ? rvb : INT_MAX);
-        }
-        if (!kMulti) {
-            __syncwarp();  // orders lane 0's shared-memory bookkeeping before other lanes read it
-            return w;
-        }
         Red *buf = sred[rb & 1];
         ++rb;
         if (lane == 0) buf[warp] = w;
@@ -266,37 +211,28 @@ struct Round {
         return w;
     }
 
-    static __device__ __forceinline__ bool block_any(bool p)
-    {
-        if (!kMulti) return __any_sync(kFull, p);
-        return __syncthreads_or(p) != 0;
-    }
+    static __device__ __forceinline__ bool block_any(bool p) { return __syncthreads_or(p) != 0; }
 
-    static __device__ __forceinline__ void sync()
-    {
-        if (kMulti) __syncthreads();
-        else __syncwarp();
-    }
+    static __device__ __forceinline__ void sync() { __syncthreads(); }
 
     enum { kUpdate = 0, kMin = 1, kStraight = 2 };
 
     // Row update for one flip: g += c * W_k* over the P slots (Eq.(16), field
     // form), then, unless kMode == kUpdate, the n neighbour deltas (Eq.(5)):
     // min over all bits (vmin) and, kMode == kStraight, over the mismatches (cmin);
-    // vj / cj: the first of this thread's byte-groups holding vmin / cmin.
+    // cj: the first of this thread's byte-groups holding cmin.
     template <int kMode>
     static __device__ __forceinline__ void process_row(int (&g)[kP], M xm, M mism, const uint4 *row4, uint64_t *bars,
-                                                       uint32_t par, int c, int t, int nt, int &vmin, int &vj,
-                                                       int &cmin, int &cj)
+                                                       uint32_t par, int c, int t, int nt, int &vmin, int &cmin,
+                                                       int &cj)
     {
         const int cb = c & 0xff;  // c = +-2 as a signed byte
         vmin = INT_MAX;
-        vj = 0;
         cmin = INT_MAX;
         cj = 0;  // kStraight: first byte-group holding cmin (lowest index, reading C5)
 #pragma unroll
         for (int j = 0; j < G; ++j) {
-            int gmin = INT_MAX, gv = INT_MAX;
+            int gmin = INT_MAX;
             if (kRowChunks == 2 ? (j % (G / 2) == 0) : (j == 0)) mbar_wait(&bars[kRowChunks == 2 ? j / (G / 2) : 0], par);
             const uint4 w4 = row4[t + nt * j];
             const uint32_t wv[4] = {w4.x, w4.y, w4.z, w4.w};
@@ -311,18 +247,13 @@ struct Round {
                 if (kMode != kUpdate) {
                     const int d0 = readout(g[s0], xm, s0);
                     const int d1 = readout(g[s0 + 1], xm, s0 + 1);
-                    if (kOwnerB) gv = min(gv, min(d0, d1));
-                    else vmin = min(vmin, min(d0, d1));
+                    vmin = min(vmin, min(d0, d1));
                     if (kMode == kStraight) {
                         const int m0 = bit(mism, s0) ? d0 : INT_MAX;
                         const int m1 = bit(mism, s0 + 1) ? d1 : INT_MAX;
                         gmin = min(gmin, min(m0, m1));
                     }
                 }
-            }
-            if (kOwnerB && kMode != kUpdate && gv < vmin) {
-                vmin = gv;
-                vj = j;
             }
             if (kMode == kStraight && gmin < cmin) {
                 cmin = gmin;
@@ -459,8 +390,8 @@ struct Round {
             // multi-warp: each warp walks only the proposals whose owner thread is one of
             // its lanes, about nb / warps of them instead of nb (random32k SA +6%, tsp100
             // +3%; one warp owns them all, and the ballot measured -2% on MaxCut there)
-            unsigned mine = nb >= 32 ? kFull : (1u << nb) - 1u;
-            if constexpr (kMulti) {
+            unsigned mine;
+            {
                 const int own = lane < nb ? (kq >> 3) - nt * group_of(kq, nt) : -1;
                 mine = __ballot_sync(kFull, lane < nb && (own >> 5) == (t >> 5));
             }
@@ -621,9 +552,9 @@ struct Round {
                 const int j = group_of(k, nt);
                 if (t == (k >> 3) - nt * j) xm ^= (M)1 << (8 * j + (k & 7));  // x_k <- 1 - x_k
             }
-            int vmin, vj, cmin, cj;
+            int vmin, cmin, cj;
             process_row<kUpdate>(g, xm, 0, reinterpret_cast<const uint4 *>(rowbuf + rowb * b), sm->bar[b], par, c, t,
-                                 nt, vmin, vj, cmin, cj);
+                                 nt, vmin, cmin, cj);
             a += l;  // offset <- (a + l) mod n
             if (a >= n) a -= n;
             int a2 = a + l;
@@ -675,7 +606,7 @@ struct Round {
     static __device__ __forceinline__ void run(const RoundArgs &A, unsigned char *smem, int sid, const uint8_t *Ts,
                                                const Out &out, int &fbase)
     {
-        const int nt = kNT ? kNT : (kMulti ? A.nt : 32);
+        const int nt = kNT ? kNT : A.nt;
         const int n = A.n;
         const int t = threadIdx.x;
         const int lane = t & 31, warp = t >> 5, nw = nt >> 5;
@@ -685,11 +616,11 @@ struct Round {
         const size_t rowb = (size_t)2 * kP * nt;  // bytes of one padded row (2 * n_pad)
 
         RoundSmem *sm = reinterpret_cast<RoundSmem *>(smem);
-        WindowSmem *win = reinterpret_cast<WindowSmem *>(smem + sizeof(RoundSmem));  // kMulti only
-        M *stm = reinterpret_cast<M *>(smem + sizeof(RoundSmem) + (kMulti ? sizeof(WindowSmem) : 0));
+        WindowSmem *win = reinterpret_cast<WindowSmem *>(smem + sizeof(RoundSmem));
+        M *stm = reinterpret_cast<M *>(smem + sizeof(RoundSmem) + sizeof(WindowSmem));
         M *sbm = stm + nt;
         unsigned char *rowbuf =
-            smem + ((sizeof(RoundSmem) + (kMulti ? sizeof(WindowSmem) : 0) + 2 * sizeof(M) * nt + 127) & ~size_t(127));
+            smem + ((sizeof(RoundSmem) + sizeof(WindowSmem) + 2 * sizeof(M) * nt + 127) & ~size_t(127));
 
         if (t == 0) {
             sm->hash = A.hash[sid];
@@ -724,7 +655,7 @@ struct Round {
         int a = A.a[sid];
         const int l = A.l[sid];
         constexpr bool sa = kSA;  // ABS_POLICY_SA: a separate kernel instantiation
-        const bool pre = kMulti && l <= kWinMax && !sa;
+        const bool pre = l <= kWinMax && !sa;
         int left = (int)A.L;
         int sa_bsz = 1;  // SA: proposals per batch (sa_next)
         int sa_cadd = 0, sa_lon = 0, sa_los = 0, sa_loq = 0;  // SA: early decision bookkeeping (sa_next)
@@ -739,12 +670,9 @@ struct Round {
             have = sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq);
         } else {
             int cv, ci2;
-            if constexpr (kMulti) {  // one inlined scan (code size of the flip loop)
+            {  // one inlined scan (code size of the flip loop)
                 const M cm = straight ? (M)(xm ^ stm[t]) : window_mask(a, l, n, t, nt);
                 candidates(g, xm, cm, t, nt, cv, ci2);
-            } else {
-                if (straight) candidates(g, xm, (M)(xm ^ stm[t]), t, nt, cv, ci2);
-                else candidates_window(g, xm, a, l, n, t, nt, cv, ci2);
             }
             if (pre && !straight) {
                 int a2 = a + l;
@@ -763,7 +691,7 @@ struct Round {
         ABS_T(if (lane == 0) for (int q = 0; q < 24; ++q) sm->tacc[warp][q] = 0;)
         for (; have; ++f) {
 #ifndef ABS_TIMING
-            if constexpr (kMulti && !kSA) {
+            if constexpr (!kSA) {
                 if (pre && !straight)
                     fast_local(A, sm, win, rowbuf, rowb, g, xm, a, l, n, t, nt, lane, warp, nw, ctl, left, k, dk, xk,
                                exact, f, fbase);
@@ -821,15 +749,15 @@ struct Round {
                 const int j = group_of(k, nt);
                 if (t == (k >> 3) - nt * j) xm ^= (M)1 << (8 * j + (k & 7));  // x_k <- 1 - x_k
             }
-            int vmin, vj, cmin, cj;
+            int vmin, cmin, cj;
             const uint4 *row4 = reinterpret_cast<const uint4 *>(row);
             M mism = 0;
             if (straight) {
                 mism = xm ^ stm[t];
-                process_row<kStraight>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, vj, cmin, cj);
+                process_row<kStraight>(g, xm, mism, row4, sm->bar[b], par, c, t, nt, vmin, cmin, cj);
             } else {
-                if (exact) process_row<kMin>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, vj, cmin, cj);
-                else process_row<kUpdate>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, vj, cmin, cj);
+                if (exact) process_row<kMin>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin, cj);
+                else process_row<kUpdate>(g, xm, 0, row4, sm->bar[b], par, c, t, nt, vmin, cmin, cj);
                 if (!sa) {
                     a += l;  // offset <- (a + l) mod n
                     if (a >= n) a -= n;
@@ -875,10 +803,8 @@ struct Round {
 
             ABS_T(long long tc4 = clock64();)
             Red r1;
-            int r1vb = INT_MAX;  // kOwnerB: byte-group of the lowest bit attaining r1.v
-            if (exact || (!kMulti && !pre)) {  // one warp: the next window argmin is reduced here too
-                r1 = block_reduce(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw,
-                                  vmin != INT_MAX ? t + nt * vj : INT_MAX, &r1vb);
+            if (exact) {
+                r1 = block_reduce(Red{vmin, cmin, ci2}, sm->red, rb, lane, warp, nw);
             } else {
                 sync();  // row buffer b free; sel[b], thr[b] and the window published
                 r1 = Red{INT_MAX, INT_MAX, INT_MAX};
@@ -900,15 +826,7 @@ struct Round {
                 const int beta = r1.i;
                 const int jb = group_of(8 * beta, nt);
                 const int owner = beta - nt * jb;
-                if (!kMulti) {
-                    if (t == owner) {
-                        snext = lowest_equal_group(g, xm, mism, r1.c, jb, t, nt);
-                        sm->snext[b] = snext;
-                        issue_row(A, snext >> 1, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
-                    }
-                    __syncwarp();
-                    snext = sm->snext[b];
-                } else if (warp == (owner >> 5)) {
+                if (warp == (owner >> 5)) {
                     if (t == owner) {
                         snext = lowest_equal_group(g, xm, mism, r1.c, jb, t, nt);
                         sm->snext[b] = snext;
@@ -925,21 +843,11 @@ struct Round {
             if (improve) {
                 M bm = xm;
                 if (r1.v < 0) {  // B = X' with its best neighbour flipped (reading C2)
-                    if constexpr (kOwnerB) {
-                        // the reduction named the lowest byte-group holding the minimum; its owner
-                        // finds the lowest bit i* in its 8 slots and flips it in its part of B
-                        const int jv = group_of(8 * r1vb, nt);
-                        if (t == r1vb - nt * jv) {
-                            const int istar = lowest_equal_group(g, xm, ~(M)0, r1.v, jv, t, nt) >> 1;
-                            bm ^= (M)1 << (8 * jv + (istar & 7));
-                        }
-                    } else {
-                        const int it = (vmin == r1.v) ? lowest_equal(g, xm, ~(M)0, r1.v, t, nt) : INT_MAX;
-                        const Red r2 = block_reduce(Red{it, INT_MAX, INT_MAX}, sm->red, rb, lane, warp, nw);
-                        const int istar = r2.v >> 1;
-                        const int j = group_of(istar, nt);
-                        if (t == (istar >> 3) - nt * j) bm ^= (M)1 << (8 * j + (istar & 7));
-                    }
+                    const int it = (vmin == r1.v) ? lowest_equal(g, xm, ~(M)0, r1.v, t, nt) : INT_MAX;
+                    const Red r2 = block_reduce(Red{it, INT_MAX, INT_MAX}, sm->red, rb, lane, warp, nw);
+                    const int istar = r2.v >> 1;
+                    const int j = group_of(istar, nt);
+                    if (t == (istar >> 3) - nt * j) bm ^= (M)1 << (8 * j + (istar & 7));
                 }
                 sbm[t] = bm;
             }
@@ -960,22 +868,10 @@ struct Round {
                         k = e.x;
                         dk = e.y;
                         xk = e.z;
-                        if constexpr (!kMulti) {
-                            __syncwarp();
-                            const long long E1 = sm->E;
-                            const long long LB2 = min(sm->LB - 2 * (long long)A.wmax, -(long long)dk);
-                            exact = E1 + dk + min(LB2, 0LL) < sm->EB;
-                        }
                         continue;
                     }
                 }
                 if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq)) break;
-                if constexpr (!kMulti) {
-                    __syncwarp();
-                    const long long E1 = sm->E;
-                    const long long LB2 = min(sm->LB - 2 * (long long)A.wmax, -(long long)dk);
-                    exact = E1 + dk + min(LB2, 0LL) < sm->EB;
-                }
             } else if (!straight) {
                 if (--left <= 0) break;
                 if (pre) {
@@ -999,14 +895,6 @@ struct Round {
                 k = r1.i >> 1;
                 xk = r1.i & 1;
                 dk = r1.c;
-                if constexpr (!kMulti) {
-                    // lazy tracking for the next flip, as on the prefetch path: exact only if
-                    // E(X'') + min(0, bound on min Delta(X'')) can beat E_B
-                    __syncwarp();  // lane 0's E / LB / E_B updates of this flip
-                    const long long E1 = sm->E;
-                    const long long LB2 = min(sm->LB - 2 * (long long)A.wmax, -(long long)dk);
-                    exact = E1 + dk + min(LB2, 0LL) < sm->EB;
-                }
             } else if (!sidx) {
                 // X = T: the straight search is over; local search from T (Step 4b)
                 straight = false;
@@ -1018,8 +906,7 @@ struct Round {
                     continue;
                 }
                 int cv, cj;
-                if constexpr (kMulti) candidates(g, xm, window_mask(a, l, n, t, nt), t, nt, cv, cj);
-                else candidates_window(g, xm, a, l, n, t, nt, cv, cj);
+                candidates(g, xm, window_mask(a, l, n, t, nt), t, nt, cv, cj);
                 if (pre) {
                     int a2 = a + l;
                     if (a2 >= n) a2 -= n;
@@ -1093,10 +980,8 @@ int launch_policy(const RoundArgs &a, cudaStream_t st, size_t smem, const AsyncA
 size_t round_smem_bytes(int32_t nt, int32_t bpt)
 {
     if (nt == 32) return round_warp_smem_bytes(32 * bpt);  // one-warp searches: abs_round_warp.cu
-    const bool multi = nt > 32;
     const size_t msz = bpt == 64 ? 8 : 4;
-    size_t s = (multi ? sizeof(RoundSmemT<kSaBatchMulti>) + sizeof(WindowSmem) : sizeof(RoundSmemT<kSaBatchOne>)) +
-               2 * msz * (size_t)nt;
+    size_t s = sizeof(RoundSmemT<kSaBatchMulti>) + sizeof(WindowSmem) + 2 * msz * (size_t)nt;
     s = (s + 127) & ~size_t(127);
     return s + 2 * (size_t)2 * bpt * nt;  // two row buffers of 2 * n_pad bytes
 }
