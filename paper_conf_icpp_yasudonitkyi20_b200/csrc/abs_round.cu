@@ -228,6 +228,7 @@ struct Round {
     {
         const int cb = c & 0xff;  // c = +-2 as a signed byte
         vmin = INT_MAX;
+        int vmin2 = INT_MAX;  // odd groups: two independent min chains (shorter dependency chain)
         cmin = INT_MAX;
         cj = 0;  // kStraight: first byte-group holding cmin (lowest index, reading C5)
 #pragma unroll
@@ -247,7 +248,8 @@ struct Round {
                 if (kMode != kUpdate) {
                     const int d0 = readout(g[s0], xm, s0);
                     const int d1 = readout(g[s0 + 1], xm, s0 + 1);
-                    vmin = min(vmin, min(d0, d1));
+                    if (j & 1) vmin2 = min(vmin2, min(d0, d1));
+                    else vmin = min(vmin, min(d0, d1));
                     if (kMode == kStraight) {
                         const int m0 = bit(mism, s0) ? d0 : INT_MAX;
                         const int m1 = bit(mism, s0 + 1) ? d1 : INT_MAX;
@@ -260,6 +262,7 @@ struct Round {
                 cj = j;
             }
         }
+        vmin = min(vmin, vmin2);
     }
 
     // 2*index + x of the lowest mismatch slot of byte-group jsel whose Delta
