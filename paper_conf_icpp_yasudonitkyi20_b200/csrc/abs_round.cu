@@ -70,6 +70,7 @@ struct RoundSmemT {
     long long nflip, nstraight;
     unsigned long long sa_ctr;  // SA: proposals drawn (Philox counter); thread 0 writes
     int sa_tau;                 // SA: this search's temperature
+    unsigned long long sa_inv;  // SA: sa_inv2tau(sa_tau)
     int sa_d[2][kB], sa_x[2][kB];  // SA: Delta_k / x_k of a batch of proposals, by batch parity
     int sa_k[2][kB];               // SA: the batch's proposed bits ...
     uint32_t sa_o[2][kB];          // ... and their acceptance draws
@@ -371,6 +372,7 @@ struct Round {
         unsigned long long c = sm->sa_ctr + (unsigned long long)cadd;
         cadd = 0;
         const int tau = sm->sa_tau;
+        const uint64_t inv2tau = sm->sa_inv;
         const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
         const int lane = t & 31;
         bool acc = false;
@@ -421,7 +423,7 @@ struct Round {
             if (lane < nb) {
                 d = sm->sa_d[sb][lane];
                 x = sm->sa_x[sb][lane];
-                ok = sa_accept(d, tau, o1);  // Eq.(7)
+                ok = sa_accept(d, tau, inv2tau, o1);  // Eq.(7)
             }
             const unsigned m = __ballot_sync(kFull, ok);
             if (m) {
@@ -634,6 +636,7 @@ struct Round {
             sm->LB = INT64_MIN / 4;
             sm->sa_ctr = A.policy == 1 ? A.sa_ctr[sid] : 0ull;
             sm->sa_tau = A.policy == 1 ? A.tau[sid] : 1;
+            sm->sa_inv = sa_inv2tau(sm->sa_tau);
         }
 
         // ---- the search state (registers for the whole round)
@@ -734,7 +737,7 @@ struct Round {
                         d = d0 + reinterpret_cast<const short *>(row)[kk] * (2 - 4 * (x0 ^ xk));
                         xn = x0;
                     }
-                    ok = sa_accept(d, sm->sa_tau, o1);  // Eq.(7)
+                    ok = sa_accept(d, sm->sa_tau, sm->sa_inv, o1);  // Eq.(7)
                 }
                 const unsigned m = __ballot_sync(kFull, ok);
                 const int j = m ? __ffs(m) - 1 : -1;

@@ -99,18 +99,24 @@ __device__ __noinline__ uint64_t sa_threshold_exact(int dE, int tau)
     return y >> (31 + q);  // 2^32 2^(-q) y / 2^63
 }
 
+// floor((2^64 - 1) / (2 tau)): sa_accept's reciprocal of the chord denominator, once per round
+__device__ __forceinline__ uint64_t sa_inv2tau(int tau) { return ~0ull / (2ull * (uint32_t)tau); }
+
 // u < P(dE, tau), deciding most draws without P: the chord C of 2^(-x) between
 // the integer exponents q and q+1 lies above the convex 2^(-x) and at most 6.2%
 // above it, so P <= C and P > 15 C / 16 - 1 (reading E2); only a
-// draw inside that band computes P.
-__device__ __forceinline__ bool sa_accept(int dE, int tau, uint32_t u)
+// draw inside that band computes P.  C is taken through the reciprocal inv2tau
+// (no division per draw): C' = floor(prod inv2tau / 2^64) lies in [C - 2, C],
+// and the band is widened by 2 to match.
+__device__ __forceinline__ bool sa_accept(int dE, int tau, uint64_t inv2tau, uint32_t u)
 {
     if (dE <= 0) return true;
     const uint32_t q = (uint32_t)dE / (uint32_t)tau;
     if (q > 32) return false;
     const uint32_t r = (uint32_t)dE - q * (uint32_t)tau;
-    const long long C = (long long)(((1ull << (32 - q)) * (2ull * (uint32_t)tau - r)) / (2ull * (uint32_t)tau));
-    if ((long long)u >= C + 16) return false;
+    const uint64_t prod = (1ull << (32 - q)) * (2ull * (uint32_t)tau - r);  // < 2^64
+    const long long C = (long long)__umul64hi(prod, inv2tau);
+    if ((long long)u >= C + 18) return false;
     if ((long long)u < C - (C >> 4) - 16) return true;
     return (uint64_t)u < sa_threshold_exact(dE, tau);
 }

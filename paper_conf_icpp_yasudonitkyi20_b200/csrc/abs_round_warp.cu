@@ -237,8 +237,8 @@ struct WarpRound {
     // (rejections do not change the state).  Returns false when the budget
     // `left` is spent without an acceptance.
     static __device__ __forceinline__ bool sa_next(const RoundArgs &A, int sid, const int (&D)[kP], M xm, int n, int t,
-                                                   int tau, unsigned long long &c, int &left, int &bsz, int &k, int &dk,
-                                                   int &xk)
+                                                   int tau, uint64_t inv2tau, unsigned long long &c, int &left, int &bsz,
+                                                   int &k, int &dk, int &xk)
     {
         const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
         while (left > 0) {
@@ -265,7 +265,7 @@ struct WarpRound {
                     xq = x;
                 }
             }
-            const bool ok = t < nb && sa_accept(dq, tau, o1);  // Eq.(7)
+            const bool ok = t < nb && sa_accept(dq, tau, inv2tau, o1);  // Eq.(7)
             const unsigned m = __ballot_sync(kFullMask, ok);
             if (m) {
                 const int q = __ffs(m) - 1;  // the first accepted proposal
@@ -331,6 +331,7 @@ struct WarpRound {
         const long long wmax2 = 2 * (long long)A.wmax;
         int left = (int)A.L;
         const int tau = kSA ? A.tau[sid] : 1;
+        const uint64_t inv2tau = kSA ? sa_inv2tau(tau) : 0ull;
         unsigned long long sa_c = kSA ? A.sa_ctr[sid] : 0ull;
         int sa_bsz = 1;
 
@@ -343,7 +344,7 @@ struct WarpRound {
             pass<kStraightOnly, false>(D, SG, nullptr, t, xm ^ tm, vmin, cK, cb);
             select(cK, cb, xm, t, k, dk, xk);
         } else if (kSA) {
-            have = sa_next(A, sid, D, xm, n, t, tau, sa_c, left, sa_bsz, k, dk, xk);
+            have = sa_next(A, sid, D, xm, n, t, tau, inv2tau, sa_c, left, sa_bsz, k, dk, xk);
         } else if (left > 0) {
             int K, b;
             window(D, a, l, n, t, K, b);
@@ -410,7 +411,7 @@ struct WarpRound {
                     straight = false;
                     if (left <= 0) break;
                     if (kSA) {
-                        if (!sa_next(A, sid, D, xm, n, t, tau, sa_c, left, sa_bsz, k, dk, xk)) break;
+                        if (!sa_next(A, sid, D, xm, n, t, tau, inv2tau, sa_c, left, sa_bsz, k, dk, xk)) break;
                     } else {
                         int K, bb;
                         window(D, a, l, n, t, K, bb);
@@ -420,7 +421,7 @@ struct WarpRound {
                 }
             } else {
                 if (kSA) {
-                    if (!sa_next(A, sid, D, xm, n, t, tau, sa_c, left, sa_bsz, k, dk, xk)) break;
+                    if (!sa_next(A, sid, D, xm, n, t, tau, inv2tau, sa_c, left, sa_bsz, k, dk, xk)) break;
                 } else {
                     a += l;  // offset <- (a + l) mod n
                     if (a >= n) a -= n;
