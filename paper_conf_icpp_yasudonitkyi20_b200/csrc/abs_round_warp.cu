@@ -4,7 +4,7 @@
 // Cnn / D / E are listed in DESIGN.md.
 //
 // The multi-warp kernel (abs_round.cu) is bound by the W-row stream; this one
-// is bound by instruction issue (W is L2-resident, 32 CTAs per SM), so its
+// is bound by instruction issue and latency (W is L2-resident, 24 CTAs per SM), so its
 // state is laid out to make every per-flip step as few warp instructions as
 // possible:
 //
