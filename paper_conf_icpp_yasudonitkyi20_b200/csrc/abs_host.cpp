@@ -511,8 +511,10 @@ static int lockstep_step(abs_ctx *c)
     c->have_results = true;
     c->rounds_done += S;
     if (!c->cfg.external_merge) {
-        // host Step 3: insert the new solutions (ascending search id)
+        // host Step 3: insert the new solutions (ascending search id); a result not better
+        // than the worst pool entry is rejected by the rule, checked first (most results)
         for (int s = 0; s < S; ++s) {
+            if (c->EB_h[s] >= c->pool.E.back() && c->pool.E.back() != kEInf) continue;
             std::memcpy(T.data(), c->B_h + (size_t)s * bpv, sizeof(uint32_t) * words);
             c->pool_inserted += c->pool.insert(T.data(), c->EB_h[s]) ? 1 : 0;
         }
@@ -608,10 +610,12 @@ static void async_consume(abs_ctx *c)
             const int s = (int)es[e];
             const uint32_t r = er[e];
             const size_t slot = (size_t)s * 2 + (r & 1);
-            std::memcpy(B.data(), c->Rb + slot * bpv, sizeof(uint32_t) * words);
             const int64_t EB = vload(c->Reb + slot);
             const uint32_t v = vload(c->rtver + slot);
-            c->pool_inserted += c->pool.insert(B.data(), EB) ? 1 : 0;  // Step 3
+            // Step 3; a result not better than the worst pool entry is rejected by the rule
+            const bool cand = EB < c->pool.E.back() || c->pool.E.back() == kEInf;
+            if (cand || c->cfg.trace) std::memcpy(B.data(), c->Rb + slot * bpv, sizeof(uint32_t) * words);
+            if (cand) c->pool_inserted += c->pool.insert(B.data(), EB) ? 1 : 0;
             if (c->cfg.trace) c->trace.push_back(TraceEntry{s, (int32_t)r, c->hist[s][v], B, EB});
             c->consumed[s] = r + 1;
             std::atomic_thread_fence(std::memory_order_release);
