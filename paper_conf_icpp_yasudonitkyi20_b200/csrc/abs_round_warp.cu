@@ -323,12 +323,16 @@ struct WarpRound {
         M bm = xm;  // Step 3, reading C4: B = C ...
         long long E = A.E[sid];
         long long EB = E;  // ... E_B = E(C) (Alg. 5)
-        long long LB = LLONG_MIN / 4;
+        // 32-bit bookkeeping of the lazy tracking: R = E_B - E(X) (<= 0) kept >= -2^30 (clamping
+        // it up only makes the test below more often true: conservative), and the lower bound
+        // LB on min_i Delta_i; kNoLB (unknown, or below -2^30) forces the next flip exact
+        constexpr int kRFloor = -(1 << 30), kNoLB = INT_MIN;
+        int R = 0, LB = kNoLB;
         unsigned long long hash = A.hash[sid];
         int nflip = 0, nstraight = 0;
         int a = A.a[sid];
         const int l = A.l[sid];
-        const long long wmax2 = 2 * (long long)A.wmax;
+        const int wmax2 = 2 * A.wmax;
         int left = (int)A.L;
         const int tau = kSA ? A.tau[sid] : 1;
         const uint64_t inv2tau = kSA ? sa_inv2tau(tau) : 0ull;
@@ -381,18 +385,21 @@ struct WarpRound {
 
             // ---- E(X') = E(X) + d_k; trajectory hash (reading D3); the bound LB
             E += dk;
+            R = max(R - dk, kRFloor);
             hash = (hash ^ (unsigned long long)(uint32_t)k) * kFnvPrimeW;
             ++nflip;
             nstraight += straight;
-            LB = min(LB - wmax2, -(long long)dk);  // Eq.(16) moves Delta_i by <= 2 wmax, Eq.(6) Delta_k -> -Delta_k
+            // Eq.(16) moves Delta_i by <= 2 wmax, Eq.(6) maps Delta_k to -Delta_k
+            LB = (LB == kNoLB || LB - wmax2 < kRFloor) ? kNoLB : min(LB - wmax2, -dk);
 
             // ---- neighbour tracking (reading C2): cand = E(X') + min(0, min_i Delta_i(X'))
             if (straight || exact) {
                 const int m = __reduce_min_sync(kFullMask, vmin >> kShift);
                 LB = m;
-                const long long cand = E + min(m, 0);
-                if (cand < EB) {
-                    EB = cand;
+                R = (int)max(EB - E, (long long)kRFloor);  // exact again (R only bounds the lazy test)
+                if (E + min(m, 0) < EB) {  // the improvement test itself in int64
+                    EB = E + min(m, 0);
+                    R = min(m, 0);
                     bm = xm;
                     if (m < 0) {  // B = X' with its best neighbour flipped
                         const int istar = lowest_equal(D, m, t);
@@ -431,8 +438,12 @@ struct WarpRound {
                     select(K, bb, xm, t, k, dk, xk);
                 }
                 // lazy tracking: exact only if E(X'') + min(0, bound on min Delta(X'')) can beat E_B
-                const long long LB2 = min(LB - wmax2, -(long long)dk);
-                exact = E + dk + min(LB2, 0LL) < EB;
+                if (LB == kNoLB || LB - wmax2 < kRFloor) {
+                    exact = true;
+                } else {
+                    const int LB2 = min(LB - wmax2, -dk);
+                    exact = dk + min(LB2, 0) < R;
+                }
             }
             if (t == 0) issue_row(A, k, rowbuf + kRowB * (b ^ 1), &sm->bar[b ^ 1]);
         }
