@@ -138,3 +138,30 @@ def test_counter_persists_across_calls():
     b.local_sa(400)
     assert a.sa_ctr == b.sa_ctr == 700
     assert a.E == b.E and a.hash == b.hash and (a.x == b.x).all() and (a.d == b.d).all()
+
+
+def test_replay_search_sa_equals_lockstep_run():
+    """oracle.replay_search with the SA policy (the async-parity reference)
+    re-runs one search of oracle.run_lockstep exactly, given the targets that
+    search received: same temperature (reading E2 ladder), same Philox stream
+    (global search id), the proposal counter persisting across rounds."""
+    n, S, L, R, seed = 120, 5, 300, 3, 21
+    tmin, tmax, K = 2000, 90000, 3
+    W = random_qubo(n, 22)
+    cfg = oracle.Config(n=n, searches=S, local_flips=L, pool_size=8, seed=seed, policy=1,
+                        sa_tau_min=tmin, sa_tau_max=tmax, sa_levels=K)
+    o = oracle.run_lockstep(W, cfg, R)
+    # the targets of rounds 0..R-1: rebuild the pool exactly as run_lockstep does
+    pool = oracle.Pool(n, 8, seed)
+    T = np.zeros((R, S, (n + 31) // 32), np.uint32)
+    for r in range(R):
+        for s in range(S):
+            T[r, s] = pool.target(cfg, r, s)
+        for s in range(S):
+            pool.insert(o["B"][r, s], o["EB"][r, s])
+    for s in range(S):
+        rep = oracle.replay_search(W, 0, L, T[:, s], policy=1, tau=oracle.sa_tau_of(s, tmin, tmax, K),
+                                   sid=s, seed=seed)
+        assert (rep["EB"] == o["EB"][:, s]).all() and (rep["B"] == o["B"][:, s]).all()
+        assert int(rep["hash"][0]) == int(o["hash"][s]) and int(rep["flips"][0]) == int(o["flips"][s])
+        assert (rep["D"] == o["D"][s]).all() and int(rep["E"][0]) == int(o["E"][s])
