@@ -3,7 +3,7 @@
 # line (with the configs 2-4 sub-results), SA lines, the reference arm, the ncu launch
 # list of the default bench command, full ncu captures of the round kernels (n = 32k
 # multi-warp, n = 1k and MaxCut n = 2000 one-warp) and of the tensor-core init kernel,
-# and compute-sanitizer runs of the one-warp kernel.  Run under gpurun; outputs in gpurun_out/.
+#.  Run under gpurun; outputs in gpurun_out/.
 set -u
 OUT=gpurun_out
 mkdir -p $OUT
@@ -26,11 +26,6 @@ timeout 900 ncu --set full --import-source on --clock-control none -k regex:roun
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:init_mma -s 2 -c 1 \
     -o $OUT/prof_init python tools/init_bench.py --n 32768 --count 1024 --engine mma --reps 2 --warmup 1 > $OUT/prof_init.log 2>&1; echo "ncu-init rc=$?"
 timeout 300 python tools/init_bench.py > $OUT/init_bench.jsonl 2>&1; echo "init-bench rc=$?"
-mkdir -p $OUT/sanitizer
-for tool in memcheck racecheck synccheck; do for n in 100 1100; do for mode in lockstep async; do for pol in window sa; do
-  timeout 240 /usr/local/cuda/bin/compute-sanitizer --tool $tool --error-exitcode 9 --print-limit 20 \
-    python tools/sanitize_run.py --n $n --mode $mode --policy $pol > $OUT/sanitizer/${tool}_n${n}_${mode}_${pol}.log 2>&1
-  echo "$tool n=$n $mode $pol rc=$?" >> $OUT/sanitizer/summary.txt
-done; done; done; done
-cat $OUT/sanitizer/summary.txt | grep -v "rc=0" ; echo "sanitizer done"
+# compute-sanitizer is closed on the GPU pool (runs under it left GPUs needing a reset); the
+# sanitizer logs of round 2 are under profiles/r02/sanitizer_r02*.
 tail -2 $OUT/pytest_gpu.log; cut -c1-300 $OUT/bench.json
