@@ -34,19 +34,15 @@ struct MaskOf<64> {
 };
 
 constexpr uint32_t kTagSA = 0x5341504Cu;  // 'SAPL'
-// SA proposals evaluated per barrier (at most; the batch adapts, sa_next), <= 32 (one lane
-// per proposal).  Multi-warp searches (n > 2048) pay a CTA barrier per batch: 32 measured
-// +9.5% at n = 32k and +1.5% at n = 10,000 over 8.  One-warp searches keep 8: their CTAs
-// are small and many per SM, so the shared-memory bytes count (16 measured -1.5% at n = 1k).
-#ifndef ABS_SA_BATCH_ONE
-#define ABS_SA_BATCH_ONE 8
-#endif
+// SA proposals evaluated per barrier by the multi-warp searches (at most; the batch
+// adapts, Round::sa_next), <= 32 (one lane per proposal): each batch pays a CTA barrier;
+// 32 measured +9.5% at n = 32k and +1.5% at n = 10,000 over 8.  One-warp searches
+// (WarpRound::sa_next) always evaluate 32 at once against their shared-memory state mirror.
 #ifndef ABS_SA_BATCH_MULTI
 #define ABS_SA_BATCH_MULTI 32
 #endif
-constexpr int kSaBatchOne = ABS_SA_BATCH_ONE, kSaBatchMulti = ABS_SA_BATCH_MULTI;
-static_assert(kSaBatchOne >= 1 && kSaBatchOne <= 32 && kSaBatchMulti >= 1 && kSaBatchMulti <= 32,
-              "one lane per proposal");
+constexpr int kSaBatchMulti = ABS_SA_BATCH_MULTI;
+static_assert(kSaBatchMulti >= 1 && kSaBatchMulti <= 32, "one lane per proposal");
 
 // Philox4x32-10 (Salmon et al., SC'11), the library's device copy (the oracle
 // has its own; both are pinned by the Random123 known-answer vectors).
@@ -119,6 +115,21 @@ __device__ __forceinline__ bool sa_accept(int dE, int tau, uint64_t inv2tau, uin
     if ((long long)u >= C + 18) return false;
     if ((long long)u < C - (C >> 4) - 16) return true;
     return (uint64_t)u < sa_threshold_exact(dE, tau);
+}
+
+// sa_accept without its exact step: 1 accept, 0 reject, 2 undecided (u inside the
+// chord band; the caller decides it with sa_threshold_exact).
+__device__ __forceinline__ int sa_accept_fast(int dE, int tau, uint64_t inv2tau, uint32_t u)
+{
+    if (dE <= 0) return 1;
+    const uint32_t q = (uint32_t)dE / (uint32_t)tau;
+    if (q > 32) return 0;
+    const uint32_t r = (uint32_t)dE - q * (uint32_t)tau;
+    const uint64_t prod = (1ull << (32 - q)) * (2ull * (uint32_t)tau - r);  // < 2^64
+    const long long C = (long long)__umul64hi(prod, inv2tau);
+    if ((long long)u >= C + 18) return 0;
+    if ((long long)u < C - (C >> 4) - 16) return 1;
+    return 2;
 }
 
 

@@ -35,6 +35,13 @@ namespace {
 
 constexpr uint64_t kFnvPrimeW = 0x100000001b3ull;
 
+#ifndef ABS_SA_SINGLE_TRIES
+#define ABS_SA_SINGLE_TRIES 1
+#endif
+#ifndef ABS_WIN_TREE64
+#define ABS_WIN_TREE64 0
+#endif
+
 template <int kP, bool kSA>
 struct WarpRound {
     static constexpr int G = kP / 8;                      // byte-groups per lane
@@ -44,15 +51,30 @@ struct WarpRound {
     static constexpr uint32_t kPos = 2u << kShift;       // multiplier byte of phi(x_i) = +1
     static constexpr uint32_t kTog = kPos ^ (256u - kPos);  // XOR turning +m into -m in a byte
     static constexpr uint32_t kTogPair = kTog | (kTog << 24);
-    static constexpr int kSaBatch = kSaBatchOne;
     using M = typename MaskOf<kP>::T;
+    // window(): the one-group branch tree (measured on for 32 bits per lane; A/B switch for 64)
+    static constexpr bool kWinTree = kP == 32 || ABS_WIN_TREE64;
+    static constexpr int kSaSingleTries = ABS_SA_SINGLE_TRIES;
 
     struct Smem {
         uint64_t bar[2];  // row buffer b completes on bar[b]
     };
     static constexpr size_t kHeader = 128;
+    // Row buffers: two (double-buffered by flip parity) for the window policy.  The SA
+    // kernel uses one (the next row is issued only after the warp has consumed the current
+    // one) and spends the bytes on a MIRROR of the state in shared memory -- every lane's
+    // keys (chunk c = slots 4c..4c+3 of lane t at ((c * 32 + t) * 16) and x bits -- so the
+    // owner of any proposed bit is one shared load away (sa_next).
+    static constexpr int kBufs = kSA ? 1 : 2;
+    static constexpr uint32_t kRowB = 2u * kP * 32;  // one row: 2 n_pad bytes
+    static constexpr size_t kMirOff = kHeader + (size_t)kBufs * kRowB;
+    static constexpr size_t kMirX = kMirOff + (size_t)kP * 32 * 4;
 
-    static __host__ __device__ size_t smem_bytes(int n_pad) { return kHeader + 2 * (size_t)2 * n_pad; }
+    static __host__ __device__ size_t smem_bytes(int n_pad)
+    {
+        (void)n_pad;  // n_pad = 32 kP
+        return kSA ? kMirX + 32 * sizeof(M) : kMirOff;
+    }
 
     static __device__ __forceinline__ void init_barriers(unsigned char *smem)
     {
@@ -72,6 +94,11 @@ struct WarpRound {
     // slot of bit i in its owner lane ((i >> 3) & 31)
     static __device__ __forceinline__ int slot_of(int i) { return ((i >> 8) << 3) | (i & 7); }
     static __device__ __forceinline__ int lane_of(int i) { return (i >> 3) & 31; }
+    static __device__ __forceinline__ int popc_m(M x)
+    {
+        if constexpr (sizeof(M) == 8) return __popcll(x);
+        else return __popc(x);
+    }
 
     // bits [lo, hi) of the byte-group starting at bit `base`, as an 8-bit mask
     static __device__ __forceinline__ uint32_t range8(int base, int lo, int hi)
@@ -145,8 +172,8 @@ struct WarpRound {
     // tracking, Eq.(5)); kUpdStraight / kStraightOnly: (cK, cb) = lowest-index
     // argmin key over the mismatches `mism` (Alg. 5).
     template <int kMode, bool kX1>
-    static __device__ __forceinline__ void pass(int (&D)[kP], const uint32_t (&SG)[kP / 2], const uint4 *row4, int t,
-                                                M mism, int &vmin, int &cK, int &cb)
+    static __device__ __forceinline__ void pass(int (&D)[kP], const uint32_t (&SG)[kP / 2], uint32_t rowl, M mism,
+                                                int &vmin, int &cK, int &cb)
     {
         vmin = INT_MAX;
         cK = INT_MAX;
@@ -155,7 +182,7 @@ struct WarpRound {
 #pragma unroll
         for (int j = 0; j < G; ++j) {
             if (kMode != kStraightOnly) {
-                const uint4 w = row4[t + 32 * j];
+                const uint4 w = lds128(rowl + 512u * j);  // rowl: this lane's 16 bytes of byte-group 0
                 const uint32_t wv[4] = {w.x, w.y, w.z, w.w};
 #pragma unroll
                 for (int q = 0; q < 4; ++q) {
@@ -179,11 +206,79 @@ struct WarpRound {
         }
     }
 
+    static __device__ __forceinline__ int min8(const int *d)
+    {
+        return min(min(min(d[0], d[1]), min(d[2], d[3])), min(min(d[4], d[5]), min(d[6], d[7])));
+    }
+
+    // Lane part of a window inside byte-group j (warp-uniform), reached by a uniform
+    // branch tree over the groups.  Aligned (byte-aligned window): K = min of the lane's 8
+    // keys of group j if its byte is inside (`in`), else INT_MAX.  Masked: K = min over the
+    // lane's bits of group j in the window [a, end) (beta: the lane's byte of group j).
+    template <int LO, int HI>
+    static __device__ __forceinline__ void win_aligned(const int (&D)[kP], int j, bool in, int &K)
+    {
+        if constexpr (HI - LO == 1) {
+            K = in ? min8(&D[8 * LO]) : INT_MAX;
+        } else {
+            constexpr int MID = (LO + HI) / 2;
+            if (j < MID) win_aligned<LO, MID>(D, j, in, K);
+            else win_aligned<MID, HI>(D, j, in, K);
+        }
+    }
+    template <int LO, int HI>
+    static __device__ __forceinline__ void win_masked(const int (&D)[kP], int j, int beta, int a, int end, int &K)
+    {
+        if constexpr (HI - LO == 1) {
+            const uint32_t m = range8(8 * beta, a, end);
+            int bk = INT_MAX;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) bk = min(bk, ((m >> e) & 1u) ? D[8 * LO + e] : INT_MAX);
+            K = bk;
+        } else {
+            constexpr int MID = (LO + HI) / 2;
+            if (j < MID) win_masked<LO, MID>(D, j, beta, a, end, K);
+            else win_masked<MID, HI>(D, j, beta, a, end, K);
+        }
+    }
+
     // Lane part of the window argmin over {(a + r) mod n : r < l} (Fig. 2, P:L305;
     // reading C6): only the byte-groups j the window touches (warp-uniform).
     static __device__ __forceinline__ void window(const int (&D)[kP], int a, int l, int n, int t, int &K, int &b)
     {
         const int end = a + l;  // exclusive; > n when the window wraps
+        if (kWinTree && end <= n && (a >> 8) == ((end - 1) >> 8)) {
+            // The common case: the window lies in ONE byte-group j0 (no wrap, l <= 256 within
+            // a 256-bit group), so only that group's 8 keys per lane are read, reached by a
+            // uniform branch tree (no per-group tests).
+            const int j0 = a >> 8;
+            const int beta = t + 32 * j0;  // this lane's byte of group j0
+            if (((a | l) & 7) == 0) win_aligned<0, G>(D, j0, (unsigned)(beta - (a >> 3)) < (unsigned)(l >> 3), K);
+            else win_masked<0, G>(D, j0, beta, a, end, K);
+            b = (8 * j0) >> kShift;
+            return;
+        }
+        if (((a | l) & 7) == 0 && end <= n) {
+            // Byte-aligned window without wrap over several groups: a lane holds whole bytes of
+            // it, so a touched byte-group contributes the min of its 8 keys or nothing.
+            const int b0 = a >> 3, nb = l >> 3;  // window bytes [b0, b0 + nb)
+            const int j0 = a >> 8, j1 = (end - 1) >> 8;
+            K = INT_MAX;
+            b = 0;
+            int bk = INT_MAX;
+#pragma unroll
+            for (int j = 0; j < G; ++j) {
+                if (j >= j0 && j <= j1) {
+                    const int gm = min8(&D[8 * j]);
+                    if ((unsigned)(t + 32 * j - b0) < (unsigned)nb) bk = min(bk, gm);
+                }
+                if (((8 * (j + 1)) & (kBlk - 1)) == 0) {
+                    if (bk != INT_MAX) combine(K, b, bk, (8 * j) >> kShift);
+                    bk = INT_MAX;
+                }
+            }
+            return;
+        }
         const int hi1 = min(end, n);
         const int hi2 = end - n;
         const int jA = a >> 8, jB = (hi1 - 1) >> 8;
@@ -222,54 +317,108 @@ struct WarpRound {
         return __reduce_min_sync(kFullMask, r);
     }
 
-    static __device__ __forceinline__ void issue_row(const RoundArgs &A, int k, unsigned char *buf, uint64_t *bar)
+    // Row k of W into the row buffer at shared address buf, completing on the
+    // mbarrier at shared address bar (one lane).
+    static __device__ __forceinline__ void issue_row(const RoundArgs &A, int k, uint32_t buf, uint32_t bar)
     {
         const uint32_t bytes = (uint32_t)(2 * kP * 32);  // 2 n_pad
-        mbar_arrive_expect_tx(bar, bytes);
-        bulk_g2s(buf, reinterpret_cast<const char *>(A.Wz) + (size_t)k * bytes, bytes, bar);
+        mbar_arrive_expect_tx_a(bar, bytes);
+        bulk_g2s_a(buf, reinterpret_cast<const char *>(A.Wz) + (size_t)k * bytes, bytes, bar);
     }
 
-    // SA policy (Alg. 1 + Eq.(7), reading E2): proposals from the search's
-    // Philox stream in batches of bsz (lane q draws proposal c + q); each
-    // proposal's Delta_k and x_k come from its owner lane; lane q decides
-    // proposal q; the first acceptance is taken and the proposals after it are
-    // drawn again after the flip, so the decisions are the one-at-a-time ones
-    // (rejections do not change the state).  Returns false when the budget
-    // `left` is spent without an acceptance.
-    static __device__ __forceinline__ bool sa_next(const RoundArgs &A, int sid, const int (&D)[kP], M xm, int n, int t,
-                                                   int tau, uint64_t inv2tau, unsigned long long &c, int &left, int &bsz,
-                                                   int &k, int &dk, int &xk)
+    // The state mirror the SA proposals read (smem_bytes): keys and x bits of every lane.
+    static __device__ __forceinline__ void mirror(unsigned char *smem, const int (&D)[kP], M xm, int t)
+    {
+        uint4 *mk = reinterpret_cast<uint4 *>(smem + kMirOff);
+#pragma unroll
+        for (int c = 0; c < kP / 4; ++c)
+            mk[c * 32 + t] = make_uint4((uint32_t)D[4 * c], (uint32_t)D[4 * c + 1], (uint32_t)D[4 * c + 2],
+                                        (uint32_t)D[4 * c + 3]);
+        reinterpret_cast<M *>(smem + kMirX)[t] = xm;
+    }
+
+    // SA policy (Alg. 1 + Eq.(7), reading E2): the next accepted proposal from
+    // the search's Philox stream (proposal c draws bit k = o0 mod n and the
+    // uniform o1), in one of two modes:
+    //  * single (`one`): proposal c alone, Delta_k and x_k fetched from the owner
+    //    lane's registers (uniform slot tree + shuffles) -- cheapest when
+    //    acceptances are frequent;
+    //  * batch: 32 proposals at once, lane q drawing and deciding proposal c + q
+    //    against the state mirror in shared memory (Delta_k and x_k of every
+    //    proposal one shared load away), written at most once per flip (`mir`).
+    // kSaSingleTries rejections in single mode switch to batch mode, an acceptance
+    // of the first proposal of a batch back.  Either way the first acceptance is taken
+    // and the proposals after it are drawn again after the flip, so the decisions
+    // are the one-at-a-time ones (rejections do not change the state).  Returns
+    // false when the budget `left` is spent without an acceptance.
+    static __device__ __forceinline__ bool sa_next(const RoundArgs &A, int sid, unsigned char *smem, const int (&D)[kP],
+                                                   M xm, int n, int t, int tau, uint64_t inv2tau, unsigned long long &c,
+                                                   int &left, bool &one, bool &mir, int &k, int &dk, int &xk)
     {
         const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
+        const int *mk = reinterpret_cast<const int *>(smem + kMirOff);
+        const M *mx = reinterpret_cast<const M *>(smem + kMirX);
+        int miss = 0;  // single-mode rejections in this call
         while (left > 0) {
-            const int nb = min(left, bsz);
-            int kq = 0;
-            uint32_t o1 = 0;
+            if (one) {
+                uint32_t o[4];
+                philox4x32_10((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
+                const int kk = (int)(o[0] % (uint32_t)n);  // "randomly select a bit" (Alg. 1)
+                const int s = slot_of(kk), own = lane_of(kk);
+                const int v = get_slot<0, kP>(D, s);
+                const int d = __shfl_sync(kFullMask, v >> kShift, own);
+                const int x = __shfl_sync(kFullMask, (int)((xm >> s) & 1u), own);
+                --left;
+                ++c;
+                if (sa_accept(d, tau, inv2tau, o[1])) {  // Eq.(7)
+                    k = kk;
+                    dk = d;
+                    xk = x;
+                    return true;
+                }
+                if (++miss >= kSaSingleTries) one = false;
+                continue;
+            }
+            if (!mir) {
+                mirror(smem, D, xm, t);
+                __syncwarp();
+                mir = true;
+            }
+            const int nb = min(left, 32);
+            int kq = 0, dq = 0, xq = 0, dec = 0;
+            uint32_t u = 0;
             if (t < nb) {
                 uint32_t o[4];
                 const unsigned long long cq = c + (unsigned long long)t;
                 philox4x32_10((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
                 kq = (int)(o[0] % (uint32_t)n);  // "randomly select a bit" (Alg. 1)
-                o1 = o[1];
+                const int s = slot_of(kq), own = lane_of(kq);
+                dq = mk[((s >> 2) * 32 + own) * 4 + (s & 3)] >> kShift;
+                xq = (int)((mx[own] >> s) & 1u);
+                u = o[1];
+                dec = sa_accept_fast(dq, tau, inv2tau, u);  // Eq.(7), most draws decided here
             }
-            int dq = 0, xq = 0;
-            for (int q = 0; q < nb; ++q) {
-                const int kk = __shfl_sync(kFullMask, kq, q);
-                const int s = slot_of(kk);
-                const int v = get_slot<0, kP>(D, s);
-                const int own = lane_of(kk);
-                const int d = __shfl_sync(kFullMask, v >> kShift, own);
-                const int x = __shfl_sync(kFullMask, (int)((xm >> s) & 1u), own);
-                if (t == q) {
-                    dq = d;
-                    xq = x;
+            const unsigned acc = __ballot_sync(kFullMask, dec == 1);
+            unsigned unk = __ballot_sync(kFullMask, dec == 2);
+            // the first proposal that accepts: walk the candidates in order; an undecided one
+            // (u inside the chord band) is settled exactly by its own lane, only when every
+            // proposal before it has rejected (the later ones do not matter)
+            int q = -1;
+            while (acc | unk) {
+                const int c1 = __ffs(acc | unk) - 1;
+                if ((acc >> c1) & 1u) {
+                    q = c1;
+                    break;
                 }
+                const bool ex = t == c1 && (uint64_t)u < sa_threshold_exact(dq, tau);
+                if (__any_sync(kFullMask, ex)) {
+                    q = c1;
+                    break;
+                }
+                unk &= unk - 1;  // c1 rejects
             }
-            const bool ok = t < nb && sa_accept(dq, tau, inv2tau, o1);  // Eq.(7)
-            const unsigned m = __ballot_sync(kFullMask, ok);
-            if (m) {
-                const int q = __ffs(m) - 1;  // the first accepted proposal
-                if (q == 0) bsz = max(1, bsz >> 1);
+            if (q >= 0) {
+                one = q == 0;
                 k = __shfl_sync(kFullMask, kq, q);
                 dk = __shfl_sync(kFullMask, dq, q);
                 xk = __shfl_sync(kFullMask, xq, q);
@@ -279,7 +428,6 @@ struct WarpRound {
             }
             left -= nb;
             c += (unsigned long long)nb;
-            bsz = min(2 * bsz, kSaBatch);
         }
         return false;
     }
@@ -289,11 +437,10 @@ struct WarpRound {
     static __device__ __forceinline__ void run(const RoundArgs &A, unsigned char *smem, int sid, const uint8_t *Ts,
                                                const Out &out, int &fbase)
     {
-        Smem *sm = reinterpret_cast<Smem *>(smem);
-        unsigned char *rowbuf = smem + kHeader;
-        constexpr size_t kRowB = (size_t)2 * kP * 32;
         const int n = A.n;
         const int t = threadIdx.x;
+        // shared-window addresses: barrier b at sbase + 8 b, row buffer b at sbase + kHeader + kRowB b
+        const uint32_t sbase = smem_u32(smem);
 
         // ---- state: keys, multipliers, bits (Step 2: target T)
         int D[kP];
@@ -329,7 +476,8 @@ struct WarpRound {
         constexpr int kRFloor = -(1 << 30), kNoLB = INT_MIN;
         int R = 0, LB = kNoLB;
         unsigned long long hash = A.hash[sid];
-        int nflip = 0, nstraight = 0;
+        // the straight phase makes exactly Hamming(C, T) flips (Alg. 5), each reducing it by one
+        const int nstraight = __reduce_add_sync(kFullMask, (unsigned)popc_m(xm ^ tm));
         int a = A.a[sid];
         const int l = A.l[sid];
         const int wmax2 = 2 * A.wmax;
@@ -337,7 +485,7 @@ struct WarpRound {
         const int tau = kSA ? A.tau[sid] : 1;
         const uint64_t inv2tau = kSA ? sa_inv2tau(tau) : 0ull;
         unsigned long long sa_c = kSA ? A.sa_ctr[sid] : 0ull;
-        int sa_bsz = 1;
+        bool sa_one = true, sa_mir = false;  // SA: single-proposal mode; mirror holds the state
 
         // ---- first selection of the round
         bool straight = __any_sync(kFullMask, xm != tm);
@@ -345,10 +493,10 @@ struct WarpRound {
         bool have = true;
         if (straight) {
             int vmin, cK, cb;
-            pass<kStraightOnly, false>(D, SG, nullptr, t, xm ^ tm, vmin, cK, cb);
+            pass<kStraightOnly, false>(D, SG, 0u, xm ^ tm, vmin, cK, cb);
             select(cK, cb, xm, t, k, dk, xk);
         } else if (kSA) {
-            have = sa_next(A, sid, D, xm, n, t, tau, inv2tau, sa_c, left, sa_bsz, k, dk, xk);
+            have = sa_next(A, sid, smem, D, xm, n, t, tau, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk);
         } else if (left > 0) {
             int K, b;
             window(D, a, l, n, t, K, b);
@@ -357,38 +505,39 @@ struct WarpRound {
             have = false;
         }
         bool exact = true;  // compute the n neighbour deltas of this flip exactly
-        if (have && t == 0) issue_row(A, k, rowbuf + kRowB * (fbase & 1), &sm->bar[fbase & 1]);
+        if (have && elect_one())
+            issue_row(A, k, sbase + kHeader + kRowB * (kBufs == 2 ? fbase & 1 : 0), sbase + 8 * (kBufs == 2 ? fbase & 1 : 0));
 
         int f = 0;
         while (have) {
-            const int b = (fbase + f) & 1;
-            const uint32_t par = (uint32_t)((fbase + f) >> 1) & 1u;
+            // buffer b of this flip and the phase parity of its barrier
+            const int b = kBufs == 2 ? (fbase + f) & 1 : 0;
+            const uint32_t par = (uint32_t)((fbase + f) >> (kBufs == 2 ? 1 : 0)) & 1u;
             ++f;
-            mbar_wait(&sm->bar[b], par);
-            const uint4 *row4 = reinterpret_cast<const uint4 *>(rowbuf + kRowB * b);
+            mbar_wait_a(sbase + 8 * b, par);
+            const uint32_t rowl = sbase + kHeader + kRowB * b + 16 * t;
 
             // ---- flip k (Alg. 4 lines P:L328-336 / Alg. 5 lines P:L371-376)
             flip_slot<0, kP>(D, SG, slot_of(k), lane_of(k) == t);
             if (lane_of(k) == t) xm ^= (M)1 << slot_of(k);
             int vmin = INT_MAX, cK = INT_MAX, cb = 0;
             if (straight) {
-                if (xk) pass<kUpdStraight, true>(D, SG, row4, t, xm ^ tm, vmin, cK, cb);
-                else pass<kUpdStraight, false>(D, SG, row4, t, xm ^ tm, vmin, cK, cb);
+                if (xk) pass<kUpdStraight, true>(D, SG, rowl, xm ^ tm, vmin, cK, cb);
+                else pass<kUpdStraight, false>(D, SG, rowl, xm ^ tm, vmin, cK, cb);
             } else if (exact) {
-                if (xk) pass<kUpdMin, true>(D, SG, row4, t, 0, vmin, cK, cb);
-                else pass<kUpdMin, false>(D, SG, row4, t, 0, vmin, cK, cb);
+                if (xk) pass<kUpdMin, true>(D, SG, rowl, 0, vmin, cK, cb);
+                else pass<kUpdMin, false>(D, SG, rowl, 0, vmin, cK, cb);
             } else {
-                if (xk) pass<kUpd, true>(D, SG, row4, t, 0, vmin, cK, cb);
-                else pass<kUpd, false>(D, SG, row4, t, 0, vmin, cK, cb);
+                if (xk) pass<kUpd, true>(D, SG, rowl, 0, vmin, cK, cb);
+                else pass<kUpd, false>(D, SG, rowl, 0, vmin, cK, cb);
             }
             __syncwarp();  // every lane is done with row buffer b before it is refilled
+            sa_mir = false;  // SA: the mirror is stale after the flip
 
             // ---- E(X') = E(X) + d_k; trajectory hash (reading D3); the bound LB
             E += dk;
             R = max(R - dk, kRFloor);
             hash = (hash ^ (unsigned long long)(uint32_t)k) * kFnvPrimeW;
-            ++nflip;
-            nstraight += straight;
             // Eq.(16) moves Delta_i by <= 2 wmax, Eq.(6) maps Delta_k to -Delta_k
             LB = (LB == kNoLB || LB - wmax2 < kRFloor) ? kNoLB : min(LB - wmax2, -dk);
 
@@ -418,7 +567,7 @@ struct WarpRound {
                     straight = false;
                     if (left <= 0) break;
                     if (kSA) {
-                        if (!sa_next(A, sid, D, xm, n, t, tau, inv2tau, sa_c, left, sa_bsz, k, dk, xk)) break;
+                        if (!sa_next(A, sid, smem, D, xm, n, t, tau, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk)) break;
                     } else {
                         int K, bb;
                         window(D, a, l, n, t, K, bb);
@@ -428,7 +577,7 @@ struct WarpRound {
                 }
             } else {
                 if (kSA) {
-                    if (!sa_next(A, sid, D, xm, n, t, tau, inv2tau, sa_c, left, sa_bsz, k, dk, xk)) break;
+                    if (!sa_next(A, sid, smem, D, xm, n, t, tau, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk)) break;
                 } else {
                     a += l;  // offset <- (a + l) mod n
                     if (a >= n) a -= n;
@@ -445,7 +594,7 @@ struct WarpRound {
                     exact = dk + min(LB2, 0) < R;
                 }
             }
-            if (t == 0) issue_row(A, k, rowbuf + kRowB * (b ^ 1), &sm->bar[b ^ 1]);
+            if (elect_one()) issue_row(A, k, sbase + kHeader + kRowB * (kBufs == 2 ? b ^ 1 : 0), sbase + 8 * (kBufs == 2 ? b ^ 1 : 0));
         }
         fbase += f;  // rows consumed in this round (none left in flight)
 
@@ -472,7 +621,7 @@ struct WarpRound {
                 *EB_out = EB;
                 A.a[sid] = a;
                 A.hash[sid] = hash;
-                A.flips[sid] += nflip;
+                A.flips[sid] += f;  // one row per flip
                 if (kSA) A.sa_ctr[sid] = sa_c;
                 A.sflips[sid] += nstraight;
             }
