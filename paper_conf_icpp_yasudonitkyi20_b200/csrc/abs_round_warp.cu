@@ -38,6 +38,9 @@ constexpr uint64_t kFnvPrimeW = 0x100000001b3ull;
 #ifndef ABS_SA_SINGLE_TRIES
 #define ABS_SA_SINGLE_TRIES 1
 #endif
+#ifndef ABS_WARP_BUFS
+#define ABS_WARP_BUFS 1
+#endif
 #ifndef ABS_WIN_TREE64
 #define ABS_WIN_TREE64 0
 #endif
@@ -65,7 +68,7 @@ struct WarpRound {
     // one) and spends the bytes on a MIRROR of the state in shared memory -- every lane's
     // keys (chunk c = slots 4c..4c+3 of lane t at ((c * 32 + t) * 16) and x bits -- so the
     // owner of any proposed bit is one shared load away (sa_next).
-    static constexpr int kBufs = kSA ? 1 : 2;
+    static constexpr int kBufs = ABS_WARP_BUFS;
     static constexpr uint32_t kRowB = 2u * kP * 32;  // one row: 2 n_pad bytes
     static constexpr size_t kMirOff = kHeader + (size_t)kBufs * kRowB;
     static constexpr size_t kMirX = kMirOff + (size_t)kP * 32 * 4;
