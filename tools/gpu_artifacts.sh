@@ -11,8 +11,10 @@ nvidia-smi > $OUT/nvsmi.txt 2>&1
 timeout 1500 python -m pytest tests -m gpu -q --timeout 900 > $OUT/pytest_gpu.log 2>&1; echo "pytest rc=$?"
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $OUT/smoke.log 2>&1; echo "smoke rc=$?"
 timeout 900 python bench.py > $OUT/bench.json 2> $OUT/bench.err; echo "bench rc=$?"
+# SA lines: 3 steps at n >= 10,000 (~0.2-0.5 s each), 30 at n <= 2048 (a step is ~2-7 ms there)
 for w in random32k random1k maxcut2k tsp100; do
-  timeout 600 python bench.py --workload $w --policy sa --steps 3 --no-e2e --no-cpu-baseline > $OUT/sa_$w.json 2>> $OUT/bench.err; echo "sa $w rc=$?"
+  case $w in random1k|maxcut2k) st=30;; *) st=3;; esac
+  timeout 600 python bench.py --workload $w --policy sa --steps $st --no-e2e --no-cpu-baseline > $OUT/sa_$w.json 2>> $OUT/bench.err; echo "sa $w rc=$?"
 done
 timeout 600 python bench.py --impl reference --steps 2 --warmup 1 > $OUT/bench_ref.json 2> $OUT/bench_ref.err; echo "ref rc=$?"
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv \
