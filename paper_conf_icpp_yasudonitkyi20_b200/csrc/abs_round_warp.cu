@@ -25,6 +25,12 @@
 //  * Bookkeeping (E, E_B, the lazy bound LB, the flip hash) lives in
 //    registers of every lane (warp-uniform values): no shared-memory round
 //    trips, no barriers.
+//  * The window argmin touches only the byte-group the window lies in (a
+//    uniform branch tree; whole-byte minima when the window is byte-aligned).
+//  * One row buffer in shared memory: the next row is issued only after the
+//    warp has consumed the current one (its selection needs the updated keys).
+//  * SA: proposals one at a time from registers, or 32 at once against a
+//    state mirror in shared memory (sa_next).
 //
 // Global state stays in the field form of abs_internal.h (g, X bytes); it is
 // converted at the start and end of each round.
