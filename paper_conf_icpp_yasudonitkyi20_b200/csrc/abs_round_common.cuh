@@ -66,6 +66,31 @@ __device__ __forceinline__ void philox4x32_10(uint32_t c0, uint32_t c1, uint32_t
     o[3] = c3;
 }
 
+// Exact unsigned 32-bit division by a divisor fixed for a round (n for the SA bit
+// draw, tau for the acceptance exponent): Granlund-Montgomery round-up multiply,
+// q = (t + ((x - t) >> s1)) >> s2 with t = umulhi(m, x), for every x < 2^32, d >= 1
+// (tests/test_udiv.py checks the same arithmetic on the host).
+struct UDiv {
+    uint32_t d, m, s1, s2;
+};
+__host__ __device__ inline UDiv make_udiv(uint32_t d)
+{
+    uint32_t l = 0;  // ceil(log2 d)
+    while (l < 32 && (1ull << l) < d) ++l;
+    UDiv r;
+    r.d = d;
+    r.m = (uint32_t)((((1ull << l) - d) << 32) / d + 1);
+    r.s1 = l < 1 ? l : 1;
+    r.s2 = l > 1 ? l - 1 : 0;
+    return r;
+}
+__device__ __forceinline__ uint32_t udiv(uint32_t x, const UDiv &v)
+{
+    const uint32_t t = __umulhi(v.m, x);
+    return (t + ((x - t) >> v.s1)) >> v.s2;
+}
+__device__ __forceinline__ uint32_t umod(uint32_t x, const UDiv &v) { return x - udiv(x, v) * v.d; }
+
 // SA acceptance (Eq.(7), reading E2): an uphill move dE > 0 is
 // accepted with p = exp(-dE/(k_B t)), k_B t = tau / ln 2, i.e. p = 2^(-dE/tau);
 // the decision is u < P for a uniform uint32 u and the Q32 integer
@@ -131,6 +156,33 @@ __device__ __forceinline__ int sa_accept_fast(int dE, int tau, uint64_t inv2tau,
     if ((long long)u < C - (C >> 4) - 16) return 1;
     return 2;
 }
+
+// The same two with the round's divisor of tau precomputed (one-warp kernels).
+__device__ __forceinline__ bool sa_accept(int dE, const UDiv &dt, uint64_t inv2tau, uint32_t u)
+{
+    if (dE <= 0) return true;
+    const uint32_t q = udiv((uint32_t)dE, dt);
+    if (q > 32) return false;
+    const uint32_t r = (uint32_t)dE - q * dt.d;
+    const uint64_t prod = (1ull << (32 - q)) * (2ull * dt.d - r);  // < 2^64
+    const long long C = (long long)__umul64hi(prod, inv2tau);
+    if ((long long)u >= C + 18) return false;
+    if ((long long)u < C - (C >> 4) - 16) return true;
+    return (uint64_t)u < sa_threshold_exact(dE, (int)dt.d);
+}
+__device__ __forceinline__ int sa_accept_fast(int dE, const UDiv &dt, uint64_t inv2tau, uint32_t u)
+{
+    if (dE <= 0) return 1;
+    const uint32_t q = udiv((uint32_t)dE, dt);
+    if (q > 32) return 0;
+    const uint32_t r = (uint32_t)dE - q * dt.d;
+    const uint64_t prod = (1ull << (32 - q)) * (2ull * dt.d - r);  // < 2^64
+    const long long C = (long long)__umul64hi(prod, inv2tau);
+    if ((long long)u >= C + 18) return 0;
+    if ((long long)u < C - (C >> 4) - 16) return 1;
+    return 2;
+}
+
 
 
 template <class R, int kThreads, int kMinBlocks>

@@ -361,7 +361,8 @@ struct WarpRound {
     // are the one-at-a-time ones (rejections do not change the state).  Returns
     // false when the budget `left` is spent without an acceptance.
     static __device__ __forceinline__ bool sa_next(const RoundArgs &A, int sid, unsigned char *smem, const int (&D)[kP],
-                                                   M xm, int n, int t, int tau, uint64_t inv2tau, unsigned long long &c,
+                                                   M xm, const UDiv &dn, int t, const UDiv &dt, uint64_t inv2tau,
+                                                   unsigned long long &c,
                                                    int &left, bool &one, bool &mir, int &k, int &dk, int &xk)
     {
         const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
@@ -372,14 +373,14 @@ struct WarpRound {
             if (one) {
                 uint32_t o[4];
                 philox4x32_10((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
-                const int kk = (int)(o[0] % (uint32_t)n);  // "randomly select a bit" (Alg. 1)
+                const int kk = (int)umod(o[0], dn);  // "randomly select a bit" (Alg. 1): o0 mod n
                 const int s = slot_of(kk), own = lane_of(kk);
                 const int v = get_slot<0, kP>(D, s);
                 const int d = __shfl_sync(kFullMask, v >> kShift, own);
                 const int x = __shfl_sync(kFullMask, (int)((xm >> s) & 1u), own);
                 --left;
                 ++c;
-                if (sa_accept(d, tau, inv2tau, o[1])) {  // Eq.(7)
+                if (sa_accept(d, dt, inv2tau, o[1])) {  // Eq.(7)
                     k = kk;
                     dk = d;
                     xk = x;
@@ -400,12 +401,12 @@ struct WarpRound {
                 uint32_t o[4];
                 const unsigned long long cq = c + (unsigned long long)t;
                 philox4x32_10((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
-                kq = (int)(o[0] % (uint32_t)n);  // "randomly select a bit" (Alg. 1)
+                kq = (int)umod(o[0], dn);  // "randomly select a bit" (Alg. 1): o0 mod n
                 const int s = slot_of(kq), own = lane_of(kq);
                 dq = mk[((s >> 2) * 32 + own) * 4 + (s & 3)] >> kShift;
                 xq = (int)((mx[own] >> s) & 1u);
                 u = o[1];
-                dec = sa_accept_fast(dq, tau, inv2tau, u);  // Eq.(7), most draws decided here
+                dec = sa_accept_fast(dq, dt, inv2tau, u);  // Eq.(7), most draws decided here
             }
             const unsigned acc = __ballot_sync(kFullMask, dec == 1);
             unsigned unk = __ballot_sync(kFullMask, dec == 2);
@@ -419,7 +420,7 @@ struct WarpRound {
                     q = c1;
                     break;
                 }
-                const bool ex = t == c1 && (uint64_t)u < sa_threshold_exact(dq, tau);
+                const bool ex = t == c1 && (uint64_t)u < sa_threshold_exact(dq, (int)dt.d);
                 if (__any_sync(kFullMask, ex)) {
                     q = c1;
                     break;
@@ -495,6 +496,7 @@ struct WarpRound {
         const uint64_t inv2tau = kSA ? sa_inv2tau(tau) : 0ull;
         unsigned long long sa_c = kSA ? A.sa_ctr[sid] : 0ull;
         bool sa_one = true, sa_mir = false;  // SA: single-proposal mode; mirror holds the state
+        const UDiv sa_dn = make_udiv(kSA ? (uint32_t)n : 1u), sa_dt = make_udiv(kSA ? (uint32_t)tau : 1u);  // SA divisors
 
         // ---- first selection of the round
         bool straight = __any_sync(kFullMask, xm != tm);
@@ -505,7 +507,7 @@ struct WarpRound {
             pass<kStraightOnly, false>(D, SG, 0u, xm ^ tm, vmin, cK, cb);
             select(cK, cb, xm, t, k, dk, xk);
         } else if (kSA) {
-            have = sa_next(A, sid, smem, D, xm, n, t, tau, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk);
+            have = sa_next(A, sid, smem, D, xm, sa_dn, t, sa_dt, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk);
         } else if (left > 0) {
             int K, b;
             window(D, a, l, n, t, K, b);
@@ -576,7 +578,7 @@ struct WarpRound {
                     straight = false;
                     if (left <= 0) break;
                     if (kSA) {
-                        if (!sa_next(A, sid, smem, D, xm, n, t, tau, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk)) break;
+                        if (!sa_next(A, sid, smem, D, xm, sa_dn, t, sa_dt, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk)) break;
                     } else {
                         int K, bb;
                         window(D, a, l, n, t, K, bb);
@@ -586,7 +588,7 @@ struct WarpRound {
                 }
             } else {
                 if (kSA) {
-                    if (!sa_next(A, sid, smem, D, xm, n, t, tau, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk)) break;
+                    if (!sa_next(A, sid, smem, D, xm, sa_dn, t, sa_dt, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk)) break;
                 } else {
                     a += l;  // offset <- (a + l) mod n
                     if (a >= n) a -= n;
