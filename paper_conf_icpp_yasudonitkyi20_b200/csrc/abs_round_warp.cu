@@ -360,27 +360,47 @@ struct WarpRound {
     // and the proposals after it are drawn again after the flip, so the decisions
     // are the one-at-a-time ones (rejections do not change the state).  Returns
     // false when the budget `left` is spent without an acceptance.
+    // The proposal cache of sa_next: lane q holds the draw of proposal pc + q (bit pk =
+    // o0 mod n, uniform po = o1); proposals depend only on their counter (Philox), so
+    // the cache stays valid across flips.
+    struct SaCache {
+        unsigned long long pc;
+        int pk;
+        uint32_t po;
+    };
+    static __device__ __forceinline__ void sa_fill(const RoundArgs &A, int sid, const UDiv &dn, int t,
+                                                   unsigned long long c0, SaCache &pr)
+    {
+        uint32_t o[4];
+        const unsigned long long cq = c0 + (unsigned long long)t;
+        philox4x32_10((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)(A.sid0 + sid), kTagSA, (uint32_t)A.seed,
+                      (uint32_t)(A.seed >> 32), o);
+        pr.pc = c0;
+        pr.pk = (int)umod(o[0], dn);  // "randomly select a bit" (Alg. 1): o0 mod n
+        pr.po = o[1];
+    }
+
     static __device__ __forceinline__ bool sa_next(const RoundArgs &A, int sid, unsigned char *smem, const int (&D)[kP],
                                                    M xm, const UDiv &dn, int t, const UDiv &dt, uint64_t inv2tau,
-                                                   unsigned long long &c,
-                                                   int &left, bool &one, bool &mir, int &k, int &dk, int &xk)
+                                                   unsigned long long &c, SaCache &pr, int &left, bool &one,
+                                                   bool &mir, int &k, int &dk, int &xk)
     {
-        const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
         const int *mk = reinterpret_cast<const int *>(smem + kMirOff);
         const M *mx = reinterpret_cast<const M *>(smem + kMirX);
         int miss = 0;  // single-mode rejections in this call
         while (left > 0) {
             if (one) {
-                uint32_t o[4];
-                philox4x32_10((uint32_t)c, (uint32_t)(c >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
-                const int kk = (int)umod(o[0], dn);  // "randomly select a bit" (Alg. 1): o0 mod n
+                if (c - pr.pc >= 32ull) sa_fill(A, sid, dn, t, c, pr);
+                const int q = (int)(c - pr.pc);
+                const int kk = __shfl_sync(kFullMask, pr.pk, q);
+                const uint32_t u = __shfl_sync(kFullMask, pr.po, q);
                 const int s = slot_of(kk), own = lane_of(kk);
                 const int v = get_slot<0, kP>(D, s);
                 const int d = __shfl_sync(kFullMask, v >> kShift, own);
                 const int x = __shfl_sync(kFullMask, (int)((xm >> s) & 1u), own);
                 --left;
                 ++c;
-                if (sa_accept(d, dt, inv2tau, o[1])) {  // Eq.(7)
+                if (sa_accept(d, dt, inv2tau, u)) {  // Eq.(7)
                     k = kk;
                     dk = d;
                     xk = x;
@@ -394,44 +414,41 @@ struct WarpRound {
                 __syncwarp();
                 mir = true;
             }
-            const int nb = min(left, 32);
-            int kq = 0, dq = 0, xq = 0, dec = 0;
-            uint32_t u = 0;
-            if (t < nb) {
-                uint32_t o[4];
-                const unsigned long long cq = c + (unsigned long long)t;
-                philox4x32_10((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
-                kq = (int)umod(o[0], dn);  // "randomly select a bit" (Alg. 1): o0 mod n
-                const int s = slot_of(kq), own = lane_of(kq);
+            if (c - pr.pc > 16ull) sa_fill(A, sid, dn, t, c, pr);  // fewer than 16 cached: a full batch
+            const int q0 = (int)(c - pr.pc);                        // lane of proposal c
+            const int nb = min(left, 32 - q0);
+            int dq = 0, xq = 0, dec = 0;
+            if (t >= q0 && t < q0 + nb) {
+                const int s = slot_of(pr.pk), own = lane_of(pr.pk);
                 dq = mk[((s >> 2) * 32 + own) * 4 + (s & 3)] >> kShift;
                 xq = (int)((mx[own] >> s) & 1u);
-                u = o[1];
-                dec = sa_accept_fast(dq, dt, inv2tau, u);  // Eq.(7), most draws decided here
+                dec = sa_accept_fast(dq, dt, inv2tau, pr.po);  // Eq.(7), most draws decided here
             }
             const unsigned acc = __ballot_sync(kFullMask, dec == 1);
             unsigned unk = __ballot_sync(kFullMask, dec == 2);
             // the first proposal that accepts: walk the candidates in order; an undecided one
             // (u inside the chord band) is settled exactly by its own lane, only when every
             // proposal before it has rejected (the later ones do not matter)
-            int q = -1;
+            int ql = -1;
             while (acc | unk) {
                 const int c1 = __ffs(acc | unk) - 1;
                 if ((acc >> c1) & 1u) {
-                    q = c1;
+                    ql = c1;
                     break;
                 }
-                const bool ex = t == c1 && (uint64_t)u < sa_threshold_exact(dq, (int)dt.d);
+                const bool ex = t == c1 && (uint64_t)pr.po < sa_threshold_exact(dq, (int)dt.d);
                 if (__any_sync(kFullMask, ex)) {
-                    q = c1;
+                    ql = c1;
                     break;
                 }
                 unk &= unk - 1;  // c1 rejects
             }
-            if (q >= 0) {
+            if (ql >= 0) {
+                const int q = ql - q0;  // proposals before the accepted one in this batch
                 one = q == 0;
-                k = __shfl_sync(kFullMask, kq, q);
-                dk = __shfl_sync(kFullMask, dq, q);
-                xk = __shfl_sync(kFullMask, xq, q);
+                k = __shfl_sync(kFullMask, pr.pk, ql);
+                dk = __shfl_sync(kFullMask, dq, ql);
+                xk = __shfl_sync(kFullMask, xq, ql);
                 left -= q + 1;
                 c += (unsigned long long)(q + 1);
                 return true;
@@ -497,6 +514,7 @@ struct WarpRound {
         unsigned long long sa_c = kSA ? A.sa_ctr[sid] : 0ull;
         bool sa_one = true, sa_mir = false;  // SA: single-proposal mode; mirror holds the state
         const UDiv sa_dn = make_udiv(kSA ? (uint32_t)n : 1u), sa_dt = make_udiv(kSA ? (uint32_t)tau : 1u);  // SA divisors
+        SaCache sa_pr{sa_c - 64, 0, 0u};  // SA: proposal cache, empty (sa_c - pc >= 32)
 
         // ---- first selection of the round
         bool straight = __any_sync(kFullMask, xm != tm);
@@ -507,7 +525,7 @@ struct WarpRound {
             pass<kStraightOnly, false>(D, SG, 0u, xm ^ tm, vmin, cK, cb);
             select(cK, cb, xm, t, k, dk, xk);
         } else if (kSA) {
-            have = sa_next(A, sid, smem, D, xm, sa_dn, t, sa_dt, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk);
+            have = sa_next(A, sid, smem, D, xm, sa_dn, t, sa_dt, inv2tau, sa_c, sa_pr, left, sa_one, sa_mir, k, dk, xk);
         } else if (left > 0) {
             int K, b;
             window(D, a, l, n, t, K, b);
@@ -578,7 +596,7 @@ struct WarpRound {
                     straight = false;
                     if (left <= 0) break;
                     if (kSA) {
-                        if (!sa_next(A, sid, smem, D, xm, sa_dn, t, sa_dt, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk)) break;
+                        if (!sa_next(A, sid, smem, D, xm, sa_dn, t, sa_dt, inv2tau, sa_c, sa_pr, left, sa_one, sa_mir, k, dk, xk)) break;
                     } else {
                         int K, bb;
                         window(D, a, l, n, t, K, bb);
@@ -588,7 +606,7 @@ struct WarpRound {
                 }
             } else {
                 if (kSA) {
-                    if (!sa_next(A, sid, smem, D, xm, sa_dn, t, sa_dt, inv2tau, sa_c, left, sa_one, sa_mir, k, dk, xk)) break;
+                    if (!sa_next(A, sid, smem, D, xm, sa_dn, t, sa_dt, inv2tau, sa_c, sa_pr, left, sa_one, sa_mir, k, dk, xk)) break;
                 } else {
                     a += l;  // offset <- (a + l) mod n
                     if (a >= n) a -= n;
