@@ -47,6 +47,25 @@ constexpr uint64_t kFnvPrimeW = 0x100000001b3ull;
 #ifndef ABS_WARP_BUFS
 #define ABS_WARP_BUFS 1
 #endif
+// Resident CTAs (one search each) per SM the register budget is sized for: window
+// policy 24 -> 80 registers per thread (32 bits per lane), 16 -> 128 (64 bits per lane);
+// the SA kernels (Philox and the acceptance arithmetic on top) 20 -> 96 and 14 -> 128.
+// Measured (A/B, 1 B200): window 20 / 28 / 32 per SM -5% / -2% / -14% at n = 1024 (28 and
+// 32 spill, MaxCut -27%); SA 20 / 14 +2-5% over 24 / 16.
+#ifndef ABS_WARP_MINB32
+#define ABS_WARP_MINB32 24
+#endif
+#ifndef ABS_WARP_MINB64
+#define ABS_WARP_MINB64 16
+#endif
+#ifndef ABS_WARP_MINB32_SA
+#define ABS_WARP_MINB32_SA 20
+#endif
+#ifndef ABS_WARP_MINB64_SA
+#define ABS_WARP_MINB64_SA 14
+#endif
+constexpr int kMinB32 = ABS_WARP_MINB32, kMinB64 = ABS_WARP_MINB64;
+constexpr int kMinB32SA = ABS_WARP_MINB32_SA, kMinB64SA = ABS_WARP_MINB64_SA;
 #ifndef ABS_WIN_TREE64
 #define ABS_WIN_TREE64 0
 #endif
@@ -663,7 +682,8 @@ template <int kP, bool kSA>
 int launch_p(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q, int *grid_out)
 {
     using R = WarpRound<kP, kSA>;
-    return launch_kernel<R, 32, kP == 32 ? 24 : 16>(a, st, R::smem_bytes(a.n_pad), q, grid_out);
+    return launch_kernel<R, 32, kP == 32 ? (kSA ? kMinB32SA : kMinB32) : (kSA ? kMinB64SA : kMinB64)>(a, st, R::smem_bytes(a.n_pad), q,
+                                                                                                 grid_out);
 }
 
 }  // namespace
@@ -672,8 +692,8 @@ size_t round_warp_smem_bytes(int32_t n_pad) { return WarpRound<32, false>::smem_
 
 int round_warp_occupancy(int32_t bpt, int *per_sm)
 {
-    if (bpt == 32) return occupancy_of<WarpRound<32, false>, 32, 24>(32, WarpRound<32, false>::smem_bytes(1024), per_sm);
-    return occupancy_of<WarpRound<64, false>, 32, 16>(32, WarpRound<64, false>::smem_bytes(2048), per_sm);
+    if (bpt == 32) return occupancy_of<WarpRound<32, false>, 32, kMinB32>(32, WarpRound<32, false>::smem_bytes(1024), per_sm);
+    return occupancy_of<WarpRound<64, false>, 32, kMinB64>(32, WarpRound<64, false>::smem_bytes(2048), per_sm);
 }
 
 int launch_round_warp(const RoundArgs &a, cudaStream_t st, const AsyncArgs *q, int *grid_out)
