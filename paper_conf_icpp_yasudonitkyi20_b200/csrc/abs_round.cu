@@ -75,6 +75,8 @@ struct RoundSmemT {
     int sa_k[2][kB];               // SA: the batch's proposed bits ...
     uint32_t sa_o[2][kB];          // ... and their acceptance draws
     int4 sa_e;                  // SA early decision of this flip: (k, Delta_k, x_k, proposals consumed)
+    int sa_ex[2];               // SA: lazy test of the early-accepted next flip (1: exact), by flip parity
+    long long sa_lz[2][3];      // SA: E(X'), E_B, bound LB after this flip's tracking, by flip parity
     int snext[2];               // straight phase: 2k + x of the next flip, from its owner thread
 #ifdef ABS_TIMING
     long long tacc[32][24];  // [warp][local 0-6 | straight 8-14 | selection sub-phases 16-20]
@@ -805,6 +807,15 @@ struct Round {
                     const long long LB2 = min(LB1 - 2 * (long long)A.wmax, -(long long)dk1);
                     sm->sel[b].w = (E1 + dk1 + min(LB2, 0LL) < EB) ? 1 : 0;
                 }
+                if (sa && !straight && sa_cnt > 0) {
+                    // SA lazy tracking, early-accepted next flip: the same test (this thread wrote
+                    // sa_e in the early decision above)
+                    const int4 e = sm->sa_e;
+                    if (e.x >= 0) {
+                        const long long LB2 = min(LB1 - 2 * (long long)A.wmax, -(long long)e.y);
+                        sm->sa_ex[b] = (E1 + e.y + min(LB2, 0LL) < EB) ? 1 : 0;
+                    }
+                }
             }
 
             ABS_T(long long tc4 = clock64();)
@@ -822,6 +833,11 @@ struct Round {
             if (t == ctl && exact) {
                 sm->LB = r1.v;
                 if (improve) sm->EB = sm->E + min(r1.v, 0);
+            }
+            if (sa && t == ctl) {  // for the lazy test after sa_next (read after its barrier)
+                sm->sa_lz[b][0] = sm->E;
+                sm->sa_lz[b][1] = sm->EB;
+                sm->sa_lz[b][2] = sm->LB;
             }
             const bool sidx = straight && r1.c != INT_MAX;
             int snext = 0;
@@ -874,10 +890,17 @@ struct Round {
                         k = e.x;
                         dk = e.y;
                         xk = e.z;
+                        exact = sm->sa_ex[b] != 0;  // lazy tracking (written before this flip's barrier)
                         continue;
                     }
                 }
                 if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq)) break;
+                {
+                    // lazy tracking of the next flip: exact only if E(X'') + min(0, bound on
+                    // min Delta(X'')) can beat E_B (sa_lz[b] written before sa_next's barrier)
+                    const long long LB2 = min(sm->sa_lz[b][2] - 2 * (long long)A.wmax, -(long long)dk);
+                    exact = sm->sa_lz[b][0] + dk + min(LB2, 0LL) < sm->sa_lz[b][1];
+                }
             } else if (!straight) {
                 if (--left <= 0) break;
                 if (pre) {
