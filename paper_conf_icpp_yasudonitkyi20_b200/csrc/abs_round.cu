@@ -115,6 +115,17 @@ struct Round {
         for (int m = 1; m < G; ++m) j += (beta >= m * nt);
         return j;
     }
+    // g[s] for a slot s uniform across the active threads (a binary tree over compile-time slots)
+    template <int LO, int HI>
+    static __device__ __forceinline__ int get_slot(const int (&g)[kP], int s)
+    {
+        if constexpr (HI - LO == 1) {
+            return g[LO];
+        } else {
+            constexpr int MID = (LO + HI) / 2;
+            return s < MID ? get_slot<LO, MID>(g, s) : get_slot<MID, HI>(g, s);
+        }
+    }
     static __device__ __forceinline__ int sext16(uint32_t w) { return (int)(short)(w & 0xffffu); }
 
     // bits [lo, hi) of the byte-group starting at element `base`, as an 8-bit mask
@@ -409,12 +420,7 @@ struct Round {
                 const int j = group_of(kk, nt);
                 if (t == (kk >> 3) - nt * j) {
                     const int e = kk & 7;
-                    int v = 0;
-#pragma unroll
-                    for (int jj = 0; jj < G; ++jj)
-#pragma unroll
-                        for (int ee = 0; ee < 8; ++ee)
-                            if (jj == j && ee == e) v = g[8 * jj + ee];
+                    const int v = get_slot<0, kP>(g, 8 * j + e);  // uniform slot: a branch tree, not 64 selects
                     sm->sa_d[sb][q] = readout(v, xm, 8 * j + e);
                     sm->sa_x[sb][q] = (int)bit(xm, 8 * j + e);
                 }
