@@ -71,6 +71,9 @@ struct RoundSmemT {
     unsigned long long sa_ctr;  // SA: proposals drawn (Philox counter); thread 0 writes
     int sa_tau;                 // SA: this search's temperature
     unsigned long long sa_inv;  // SA: sa_inv2tau(sa_tau)
+    UDiv sa_dn, sa_dt;          // SA: exact division by n (bit draw) and by tau (exponent), per round
+    int sa_pk[64];              // SA proposal cache: bit and draw of proposal pcb + i (sa_next)
+    uint32_t sa_po[64];
     int sa_d[2][kB], sa_x[2][kB];  // SA: Delta_k / x_k of a batch of proposals, by batch parity
     int sa_k[2][kB];               // SA: the batch's proposed bits ...
     uint32_t sa_o[2][kB];          // ... and their acceptance draws
@@ -372,7 +375,7 @@ struct Round {
     // flip's early decision; cadd counts proposals that decision consumed.
     static __device__ __forceinline__ bool sa_next(const RoundArgs &A, RoundSmem *sm, const int (&g)[kP], M xm,
                                                    int sid, int n, int t, int nt, int &left, int &k, int &dk, int &xk,
-                                                   int &bsz, int &cadd, int &lo_n, int &lo_s, int &lo_q)
+                                                   int &bsz, int &cadd, int &lo_n, int &lo_s, int &lo_q, uint32_t &pcb)
     {
         lo_n = 0;
         if (left <= 0) {  // budget spent (by the early decision): only thread 0 touches sa_ctr
@@ -384,22 +387,33 @@ struct Round {
         // once, so its barrier orders every thread's read here before thread 0's write below
         unsigned long long c = sm->sa_ctr + (unsigned long long)cadd;
         cadd = 0;
-        const int tau = sm->sa_tau;
         const uint64_t inv2tau = sm->sa_inv;
-        const uint32_t k0 = (uint32_t)A.seed, k1 = (uint32_t)(A.seed >> 32);
         const int lane = t & 31;
         bool acc = false;
         int sb = 0;  // batch slot parity (a barrier separates this call from the previous one)
         while (left > 0) {
             const int nb = min(left, bsz);
+            // proposals are drawn 64 at a time into a shared cache (two warps, one Philox per
+            // thread; proposals depend only on their counter), instead of by every warp per batch;
+            // pcb (the cache's first counter, low 32 bits) is kept by every thread in a register
+            if ((uint32_t)c - pcb + (uint32_t)nb > 64u) {
+                if (t < 64) {
+                    uint32_t o[4];
+                    const unsigned long long cq = c + (unsigned long long)t;
+                    philox4x32_10((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)(A.sid0 + sid), kTagSA,
+                                  (uint32_t)A.seed, (uint32_t)(A.seed >> 32), o);
+                    sm->sa_pk[t] = (int)umod(o[0], sm->sa_dn);  // "randomly select a bit" (Alg. 1): o0 mod n
+                    sm->sa_po[t] = o[1];
+                }
+                pcb = (uint32_t)c;
+                sync();
+            }
+            const int off = (int)((uint32_t)c - pcb);
             int kq = 0;
             uint32_t o1 = 0;
             if (lane < nb) {
-                uint32_t o[4];
-                const unsigned long long cq = c + (unsigned long long)lane;
-                philox4x32_10((uint32_t)cq, (uint32_t)(cq >> 32), (uint32_t)(A.sid0 + sid), kTagSA, k0, k1, o);
-                kq = (int)(o[0] % (uint32_t)n);  // "randomly select a bit" (Alg. 1)
-                o1 = o[1];
+                kq = sm->sa_pk[off + lane];
+                o1 = sm->sa_po[off + lane];
                 if (t < 32) {
                     sm->sa_k[sb][lane] = kq;
                     sm->sa_o[sb][lane] = o1;
@@ -431,7 +445,7 @@ struct Round {
             if (lane < nb) {
                 d = sm->sa_d[sb][lane];
                 x = sm->sa_x[sb][lane];
-                ok = sa_accept(d, tau, inv2tau, o1);  // Eq.(7)
+                ok = sa_accept(d, sm->sa_dt, inv2tau, o1);  // Eq.(7)
             }
             const unsigned m = __ballot_sync(kFull, ok);
             if (m) {
@@ -645,6 +659,8 @@ struct Round {
             sm->sa_ctr = A.policy == 1 ? A.sa_ctr[sid] : 0ull;
             sm->sa_tau = A.policy == 1 ? A.tau[sid] : 1;
             sm->sa_inv = sa_inv2tau(sm->sa_tau);
+            sm->sa_dn = make_udiv((uint32_t)A.n);
+            sm->sa_dt = make_udiv((uint32_t)sm->sa_tau);
         }
 
         // ---- the search state (registers for the whole round)
@@ -673,6 +689,7 @@ struct Round {
         int left = (int)A.L;
         int sa_bsz = 1;  // SA: proposals per batch (sa_next)
         int sa_cadd = 0, sa_lon = 0, sa_los = 0, sa_loq = 0;  // SA: early decision bookkeeping (sa_next)
+        uint32_t sa_pcb = (uint32_t)A.sa_ctr[sid] - 1000u;        // SA: proposal cache base (empty)
         int rb = 0;
         sync();
 
@@ -681,7 +698,7 @@ struct Round {
         int k = 0, dk = 0, xk = 0;
         bool have = true;  // a first flip exists (SA may accept nothing)
         if (sa && !straight) {
-            have = sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq);
+            have = sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq, sa_pcb);
         } else {
             int cv, ci2;
             {  // one inlined scan (code size of the flip loop)
@@ -745,7 +762,7 @@ struct Round {
                         d = d0 + reinterpret_cast<const short *>(row)[kk] * (2 - 4 * (x0 ^ xk));
                         xn = x0;
                     }
-                    ok = sa_accept(d, sm->sa_tau, sm->sa_inv, o1);  // Eq.(7)
+                    ok = sa_accept(d, sm->sa_dt, sm->sa_inv, o1);  // Eq.(7)
                 }
                 const unsigned m = __ballot_sync(kFull, ok);
                 const int j = m ? __ffs(m) - 1 : -1;
@@ -900,7 +917,7 @@ struct Round {
                         continue;
                     }
                 }
-                if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq)) break;
+                if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq, sa_pcb)) break;
                 {
                     // lazy tracking of the next flip: exact only if E(X'') + min(0, bound on
                     // min Delta(X'')) can beat E_B (sa_lz[b] written before sa_next's barrier)
@@ -935,7 +952,7 @@ struct Round {
                 straight = false;
                 if (left <= 0) break;
                 if (sa) {
-                    if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq)) break;
+                    if (!sa_next(A, sm, g, xm, sid, n, t, nt, left, k, dk, xk, sa_bsz, sa_cadd, sa_lon, sa_los, sa_loq, sa_pcb)) break;
                     exact = true;
                     if (t == ctl) issue_row(A, k, rowbuf + rowb * (b ^ 1), sm->bar[b ^ 1], nt);
                     continue;
