@@ -34,6 +34,8 @@
 //
 // Global state stays in the field form of abs_internal.h (g, X bytes); it is
 // converted at the start and end of each round.
+#include <type_traits>
+
 #include "abs_round_common.cuh"
 
 namespace absb {
@@ -48,12 +50,15 @@ constexpr uint64_t kFnvPrimeW = 0x100000001b3ull;
 #define ABS_WARP_BUFS 1
 #endif
 // Resident CTAs (one search each) per SM the register budget is sized for: window
-// policy 24 -> 80 registers per thread (32 bits per lane), 16 -> 128 (64 bits per lane);
-// the SA kernels (Philox and the acceptance arithmetic on top) 20 -> 96 and 14 -> 128.
-// Measured (A/B, 1 B200): window 20 / 28 / 32 per SM -5% / -2% / -14% at n = 1024 (28 and
-// 32 spill, MaxCut -27%); SA 20 / 14 +2-5% over 24 / 16.
+// policy 32 -> 64 registers per thread (32 bits per lane; fits with the multipliers in
+// shared memory, kSgSmem), 16 -> 128 (64 bits per lane); the SA kernels (Philox and the
+// acceptance arithmetic on top, multipliers in registers) 20 -> 96 and 14 -> 128.
+// Measured (A/B, 1 B200): with the multipliers in registers, window 20 / 28 / 32 per SM
+// -5% / -2% / -14% against 24 at n = 1024 (28 and 32 spill); with them in shared memory 32
+// per SM +4.5% (no spill) and 28 -7%; for 64 bits per lane 16 +4.6%, 20 -12%; SA 20 / 14
+// +2-5% over 24 / 16.
 #ifndef ABS_WARP_MINB32
-#define ABS_WARP_MINB32 24
+#define ABS_WARP_MINB32 32
 #endif
 #ifndef ABS_WARP_MINB64
 #define ABS_WARP_MINB64 16
@@ -66,6 +71,9 @@ constexpr uint64_t kFnvPrimeW = 0x100000001b3ull;
 #endif
 constexpr int kMinB32 = ABS_WARP_MINB32, kMinB64 = ABS_WARP_MINB64;
 constexpr int kMinB32SA = ABS_WARP_MINB32_SA, kMinB64SA = ABS_WARP_MINB64_SA;
+#ifndef ABS_SG_SMEM
+#define ABS_SG_SMEM 1
+#endif
 #ifndef ABS_WIN_TREE64
 #define ABS_WIN_TREE64 0
 #endif
@@ -83,6 +91,8 @@ struct WarpRound {
     // window(): the one-group branch tree (measured on for 32 bits per lane; A/B switch for 64)
     static constexpr bool kWinTree = kP == 32 || ABS_WIN_TREE64;
     static constexpr int kSaSingleTries = ABS_SA_SINGLE_TRIES;
+    // the multipliers (SG) in shared memory instead of registers (window kernels; A/B switch)
+    static constexpr bool kSgSmem = ABS_SG_SMEM && !kSA;
 
     struct Smem {
         uint64_t bar[2];  // row buffer b completes on bar[b]
@@ -98,11 +108,35 @@ struct WarpRound {
     static constexpr size_t kMirOff = kHeader + (size_t)kBufs * kRowB;
     static constexpr size_t kMirX = kMirOff + (size_t)kP * 32 * 4;
 
+    static constexpr size_t kSgOff = kSA ? kMirX + 32 * sizeof(M) : kMirOff;  // SG chunks (kSgSmem)
     static __host__ __device__ size_t smem_bytes(int n_pad)
     {
         (void)n_pad;  // n_pad = 32 kP
-        return kSA ? kMirX + 32 * sizeof(M) : kMirOff;
+        return kSgOff + (kSgSmem ? (size_t)kP / 2 * 32 * 4 : 0);
     }
+
+    // The packed multipliers of a lane: 16 (32) registers, or chunks of four in shared memory
+    // (pairs 4c..4c+3 of lane t at kSgOff + (c * 32 + t) * 16, conflict-free).
+    struct SgReg {
+        uint32_t v[kP / 2];
+        __device__ __forceinline__ uint4 chunk(int c) const
+        {
+            return make_uint4(v[4 * c], v[4 * c + 1], v[4 * c + 2], v[4 * c + 3]);
+        }
+        __device__ __forceinline__ void tog(int p, uint32_t m) { v[p] ^= m; }
+        __device__ __forceinline__ void set(int p, uint32_t m) { v[p] = m; }
+    };
+    struct SgSmem {
+        uint32_t a;  // this lane's chunk 0
+        __device__ __forceinline__ uint4 chunk(int c) const { return lds128(a + 512u * c); }
+        __device__ __forceinline__ void tog(int p, uint32_t m)
+        {
+            const uint32_t ad = a + 512u * (p >> 2) + 4u * (p & 3);
+            sts32(ad, lds32(ad) ^ m);
+        }
+        __device__ __forceinline__ void set(int p, uint32_t m) { sts32(a + 512u * (p >> 2) + 4u * (p & 3), m); }
+    };
+    using Sg = typename std::conditional<kSgSmem, SgSmem, SgReg>::type;
 
     static __device__ __forceinline__ void init_barriers(unsigned char *smem)
     {
@@ -140,12 +174,12 @@ struct WarpRound {
     // warp-uniform; a binary search over compile-time slots, nothing indexed
     // dynamically).
     template <int LO, int HI>
-    static __device__ __forceinline__ void flip_slot(int (&D)[kP], uint32_t (&SG)[kP / 2], int s, bool own)
+    static __device__ __forceinline__ void flip_slot(int (&D)[kP], Sg &SG, int s, bool own)
     {
         if constexpr (HI - LO == 1) {
             if (own) {
                 D[LO] = 2 * code_of(LO) - D[LO];
-                SG[LO >> 1] ^= (LO & 1) ? (kTog << 24) : kTog;
+                SG.tog(LO >> 1, (LO & 1) ? (kTog << 24) : kTog);
             }
         } else {
             constexpr int MID = (LO + HI) / 2;
@@ -200,7 +234,7 @@ struct WarpRound {
     // tracking, Eq.(5)); kUpdStraight / kStraightOnly: (cK, cb) = lowest-index
     // argmin key over the mismatches `mism` (Alg. 5).
     template <int kMode, bool kX1>
-    static __device__ __forceinline__ void pass(int (&D)[kP], const uint32_t (&SG)[kP / 2], uint32_t rowl, M mism,
+    static __device__ __forceinline__ void pass(int (&D)[kP], const Sg &SG, uint32_t rowl, M mism,
                                                 int &vmin, int &cK, int &cb)
     {
         vmin = INT_MAX;
@@ -212,9 +246,11 @@ struct WarpRound {
             if (kMode != kStraightOnly) {
                 const uint4 w = lds128(rowl + 512u * j);  // rowl: this lane's 16 bytes of byte-group 0
                 const uint32_t wv[4] = {w.x, w.y, w.z, w.w};
+                const uint4 m4 = SG.chunk(j);
+                const uint32_t mv[4] = {m4.x, m4.y, m4.z, m4.w};
 #pragma unroll
                 for (int q = 0; q < 4; ++q) {
-                    const uint32_t sg = kX1 ? (SG[4 * j + q] ^ kTogPair) : SG[4 * j + q];
+                    const uint32_t sg = kX1 ? (mv[q] ^ kTogPair) : mv[q];
                     D[8 * j + 2 * q] = __dp2a_lo((int)wv[q], (int)sg, D[8 * j + 2 * q]);
                     D[8 * j + 2 * q + 1] = __dp2a_hi((int)wv[q], (int)sg, D[8 * j + 2 * q + 1]);
                 }
@@ -490,7 +526,8 @@ struct WarpRound {
 
         // ---- state: keys, multipliers, bits (Step 2: target T)
         int D[kP];
-        uint32_t SG[kP / 2];
+        Sg SG;
+        if constexpr (kSgSmem) SG.a = sbase + (uint32_t)kSgOff + 16u * t;
         M xm = 0, tm = 0;
         {
             const uint8_t *Xs = A.X + (size_t)sid * G * 32;
@@ -510,7 +547,7 @@ struct WarpRound {
             for (int p = 0; p < kP / 2; ++p) {
                 const uint32_t m0 = ((xm >> (2 * p)) & 1u) ? 256u - kPos : kPos;
                 const uint32_t m1 = ((xm >> (2 * p + 1)) & 1u) ? 256u - kPos : kPos;
-                SG[p] = m0 | (m1 << 24);
+                SG.set(p, m0 | (m1 << 24));
             }
         }
         M bm = xm;  // Step 3, reading C4: B = C ...
