@@ -160,6 +160,12 @@ struct abs_ctx {
     int device = 0;
     cudaStream_t st = nullptr;
     cudaEvent_t ev0 = nullptr, ev1 = nullptr, evs0 = nullptr, evs1 = nullptr;
+    // lockstep steps of one-warp searches with more searches than resident CTAs: the
+    // first `split` searches run on st while the host builds the others' targets, which
+    // then run on st2 (their CTAs fill SMs as the first launch's finish); evj joins st2
+    cudaStream_t st2 = nullptr;
+    cudaEvent_t evj = nullptr;
+    int split = 0;
     Instance I;
     SearchState S;
     int64_t L = 0;
@@ -239,6 +245,8 @@ static void free_ctx(abs_ctx *c)
     cudaFree(c->queue_d);
     cudaFree(c->timing_d);
     cudaFree(c->done_d);
+    if (c->evj) cudaEventDestroy(c->evj);
+    if (c->st2) cudaStreamDestroy(c->st2);
     if (c->ev0) cudaEventDestroy(c->ev0);
     if (c->ev1) cudaEventDestroy(c->ev1);
     if (c->evs0) cudaEventDestroy(c->evs0);
@@ -344,6 +352,8 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
     } while (0)
 
     CTX_CU(cudaStreamCreateWithFlags(&c->st, cudaStreamNonBlocking));
+    CTX_CU(cudaStreamCreateWithFlags(&c->st2, cudaStreamNonBlocking));
+    CTX_CU(cudaEventCreateWithFlags(&c->evj, cudaEventDisableTiming));
     CTX_CU(cudaEventCreate(&c->ev0));
     CTX_CU(cudaEventCreate(&c->ev1));
     CTX_CU(cudaEventCreate(&c->evs0));
@@ -438,6 +448,13 @@ static int create_common(abs_ctx **out, int32_t n, const int16_t *W, bool W_on_d
     }
     CTX_CU(cudaMemsetAsync(S.T, 0, Sn * c->bytes_per_vec, c->st));
     CTX_CU(cudaMallocHost(&c->T_h, Sn * c->bytes_per_vec));
+    if (I.nt == 32) {  // one-warp searches: split a lockstep step beyond the resident CTAs (lockstep_step)
+        int per_sm = 0, sms = 0;
+        CTX_CU((cudaError_t)round_occupancy(I.nt, I.bpt, &per_sm));
+        CTX_CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, c->device));
+        const int resident = per_sm * sms;
+        c->split = (resident > 0 && S.S > resident) ? resident : 0;
+    }
     CTX_CU(cudaMallocHost(&c->B_h, Sn * c->bytes_per_vec));
     CTX_CU(cudaMallocHost(&c->EB_h, Sn * sizeof(int64_t)));
     std::memset(c->T_h, 0, Sn * c->bytes_per_vec);
@@ -458,12 +475,22 @@ static int lockstep_step(abs_ctx *c)
     // host Step 4: "generates ... new target solutions by GA"; the targets are
     // independent given the pool, so large batches are built on several host threads
     std::vector<uint32_t> T(words);
-    parallel_for(S, 512, [&](int s) {  // T_h rows: bpv = n_pad / 8 bytes, 4-byte aligned
-        ga_target(c->pool, c->ga, c->round, (int64_t)c->cfg.search_offset + s,
-                  reinterpret_cast<uint32_t *>(c->T_h + (size_t)s * bpv));
-    });
-    ABS_CU(cudaMemcpyAsync(c->S.T, c->T_h, (size_t)S * bpv, cudaMemcpyHostToDevice, c->st));
-    c->h2d += (int64_t)S * bpv;
+    // targets of searches [s0, s1) into T_h, then to the device on stream st
+    auto targets = [&](int s0, int s1, cudaStream_t st) -> int {
+        parallel_for(s1 - s0, 512, [&](int i) {  // T_h rows: bpv = n_pad / 8 bytes, 4-byte aligned
+            const int s = s0 + i;
+            ga_target(c->pool, c->ga, c->round, (int64_t)c->cfg.search_offset + s,
+                      reinterpret_cast<uint32_t *>(c->T_h + (size_t)s * bpv));
+        });
+        ABS_CU(cudaMemcpyAsync(c->S.T + (size_t)s0 * bpv, c->T_h + (size_t)s0 * bpv, (size_t)(s1 - s0) * bpv,
+                               cudaMemcpyHostToDevice, st));
+        c->h2d += (int64_t)(s1 - s0) * bpv;
+        return ABS_OK;
+    };
+    // one launch, or (c->split) the first `split` searches launched while the host builds the
+    // other targets: the same round for every search, the results inserted after both
+    const int s_first = c->split > 0 ? c->split : S;
+    if (const int rc = targets(0, s_first, c->st)) return rc;
     RoundArgs a{};
     a.Wz = c->I.Wz;
     a.wmax = c->I.wmax;
@@ -497,9 +524,20 @@ static int lockstep_step(abs_ctx *c)
     a.timing = c->timing_d;
 #endif
     ABS_CU(cudaEventRecord(c->ev0, c->st));
+    a.S = s_first;
+    a.sbase = 0;
     ABS_CK(launch_round(a, c->st));
     c->launches++;
     c->round_launches++;
+    if (s_first < S) {
+        if (const int rc = targets(s_first, S, c->st2)) return rc;  // overlaps the first launch
+        a.S = S - s_first;
+        a.sbase = s_first;
+        ABS_CK(launch_round(a, c->st2));
+        c->launches++;
+        ABS_CU(cudaEventRecord(c->evj, c->st2));
+        ABS_CU(cudaStreamWaitEvent(c->st, c->evj, 0));
+    }
     ABS_CU(cudaEventRecord(c->ev1, c->st));
     ABS_CU(cudaMemcpyAsync(c->B_h, c->S.B, (size_t)S * bpv, cudaMemcpyDeviceToHost, c->st));
     ABS_CU(cudaMemcpyAsync(c->EB_h, c->S.EB, (size_t)S * sizeof(int64_t), cudaMemcpyDeviceToHost, c->st));

@@ -71,6 +71,7 @@ struct RoundArgs {
     int64_t *flips, *sflips;
     int64_t L;
     int32_t S;
+    int32_t sbase;           // lockstep: search id of CTA 0 (a launch may cover searches [sbase, sbase + S))
     int32_t policy;          // ABS_POLICY_WINDOW / ABS_POLICY_SA
     int32_t sid0;            // global id of search 0 (Philox counter word)
     uint64_t seed;           // Philox key

@@ -189,7 +189,7 @@ template <class R, int kThreads, int kMinBlocks>
 __global__ void __launch_bounds__(kThreads, kMinBlocks) round_kernel(const RoundArgs A)
 {
     extern __shared__ __align__(128) unsigned char smem[];
-    const int sid = blockIdx.x;
+    const int sid = blockIdx.x + A.sbase;
     const size_t bpv = (size_t)A.n_pad / 8;
     int fbase = 0;
     R::init_barriers(smem);
