@@ -535,6 +535,7 @@ static int lockstep_step(abs_ctx *c)
         a.sbase = s_first;
         ABS_CK(launch_round(a, c->st2));
         c->launches++;
+        c->round_launches++;
         ABS_CU(cudaEventRecord(c->evj, c->st2));
         ABS_CU(cudaStreamWaitEvent(c->st, c->evj, 0));
     }

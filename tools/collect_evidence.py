@@ -13,7 +13,7 @@ with open(f"{P}/{tag}_sa_bench.jsonl", "w") as f:
     for w in ["random32k", "random1k", "maxcut2k", "tsp100"]:
         f.write(open(f"{G}/sa_{w}.json").read().strip().splitlines()[-1] + "\n")
 cases = [("prof_round", 32768, "n32k", "--n 32768 --searches 592 --steps 3 (launch 2; config 5)"),
-         ("prof_round1k", 1024, "n1k", "--n 1024 --searches 10000 --steps 3 (launch 2; config 2; WarpRound<32>)"),
+         ("prof_round1k", 1024, "n1k", "--n 1024 --searches 4736 --steps 3 (launch 2; config 2 at one launch per step: 32 x 148 resident searches; WarpRound<32>)"),
          ("prof_round2k", 2000, "maxcut2k", "--n 2000 --searches 2368 --steps 3 --workload maxcut (launch 2; config 3; WarpRound<64>)")]
 for rep, n, name, src in cases:
     fl = [json.loads(l) for l in open(f"{G}/{rep}.log") if l.startswith('{"flips"')]

@@ -22,7 +22,7 @@ timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --lo
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:round_kernel -s 2 -c 1 \
     -o $OUT/prof_round python tools/prof_round.py --n 32768 --searches 592 --steps 3 > $OUT/prof_round.log 2>&1; echo "ncu-full rc=$?"
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:round_kernel -s 2 -c 1 \
-    -o $OUT/prof_round1k python tools/prof_round.py --n 1024 --searches 10000 --steps 3 > $OUT/prof_round1k.log 2>&1; echo "ncu-full-1k rc=$?"
+    -o $OUT/prof_round1k python tools/prof_round.py --n 1024 --searches 4736 --steps 3 > $OUT/prof_round1k.log 2>&1; echo "ncu-full-1k rc=$?"
 timeout 900 ncu --set full --import-source on --clock-control none -k regex:round_kernel -s 2 -c 1 \
     -o $OUT/prof_round2k python tools/prof_round.py --n 2000 --searches 2368 --steps 3 --workload maxcut > $OUT/prof_round2k.log 2>&1; echo "ncu-full-2k rc=$?"
 timeout 600 ncu --set full --import-source on --clock-control none -k regex:init_mma -s 2 -c 1 \
