@@ -4,7 +4,7 @@
 // Cnn / D / E are listed in DESIGN.md.
 //
 // The multi-warp kernel (abs_round.cu) is bound by the W-row stream; this one
-// is bound by instruction issue and latency (W is L2-resident, 24 CTAs per SM), so its
+// is bound by instruction issue and latency (W is L2-resident, 32 CTAs per SM for 32 bits per lane, 16 for 64), so its
 // state is laid out to make every per-flip step as few warp instructions as
 // possible:
 //
@@ -18,9 +18,11 @@
 //    bookkeeping, no masks of equal values.
 //  * The flip update (Eq.(16)) Delta_i += 2 W_ik phi(x_i) phi(x_k) becomes
 //    D_s += W_ik * (2^(kShift+1) phi(x_i)) * phi(x_k): one IDP.2A per bit, the
-//    per-bit factor taken from a packed multiplier register per pair of slots
+//    per-bit factor taken from a packed multiplier word per pair of slots
 //    (byte 0: slot 2p, byte 3: slot 2p+1; dp2a.lo / dp2a.hi select them), the
-//    sign phi(x_k) applied by one XOR per pair on flips of a set bit.
+//    sign phi(x_k) applied by one XOR per pair on flips of a set bit.  The
+//    window kernels keep the multiplier words in shared memory (Sg), read next
+//    to the row, so a search fits 64 registers.
 //  * Delta_k -> -Delta_k (Eq.(6)) is D_k -> 2 (s mod 2^kShift) - D_k.
 //  * Bookkeeping (E, E_B, the lazy bound LB, the flip hash) lives in
 //    registers of every lane (warp-uniform values): no shared-memory round
