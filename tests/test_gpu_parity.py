@@ -141,6 +141,19 @@ def test_lockstep_random_qubo_bitexact(n, S, L, R, seed):
     assert_same(s, o, gB, gEB, S, n, 8)
 
 
+@pytest.mark.parametrize("n,extra,L,seed", [(40, 77, 24, 11), (1100, 33, 24, 12)])
+def test_lockstep_split_step_full_state(n, extra, L, seed):
+    """More one-warp searches than resident CTAs: a lockstep step is two launches (the
+    first resident batch, then the rest on a second stream while the host builds their
+    targets; DESIGN 5.7).  Every search's full state, every emitted result and the pool
+    equal oracle.run_lockstep, so the split is the same round for every search."""
+    S = abs_b200.device_searches(n) + extra
+    W = random_qubo(n, seed)
+    s, o, gB, gEB, gT = run_both(W, S, L, 2, pool=16, seed=seed)
+    assert s.stats()["round_kernel_launches"] == 4  # two steps, two launches each
+    assert_same(s, o, gB, gEB, S, n, 16)
+
+
 def test_lockstep_maxcut_ties_bitexact():
     # Max-Cut (Eq.(17)) with +-1 weights: deltas tie constantly -> exercises
     # the lowest-index tie-break in every reduction (reading C5).
